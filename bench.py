@@ -1,0 +1,341 @@
+#!/usr/bin/env python
+"""Benchmark: pose energy+gradient evaluations per second of the ADADELTA local
+search (BASELINE.json metric) on the drug-like workload (config 2: 40 atoms,
+8 torsions, 60^3 grid, 20 runs x 150 pop x 300 iterations = 9.0e5 evals per
+GPU per step), plus max |dE| vs the FP64 oracle.
+
+One step = one whole hot-path pass: restore the start genotypes (D2D), one
+ad_local_search call (ADADELTA kernel + best-of-run kernel), and for N > 1 the
+NCCL all_gather of the best-pose records.  Weak scaling: every rank runs its own
+config-2 replica (seed = 2000 + rank).  L2 is flushed (256 MiB write) between
+timed steps, outside the timed events.
+
+Usage: python bench.py [--gpus N] [--steps K] [--warmup W] [--engine simt|tc|paper]
+       python bench.py --impl reference ...   (times the FP64 oracle on host cores)
+Under torchrun (N > 1) every rank runs; rank 0 prints ONE JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "pose energy+gradient evals/sec (1/2/4/8 B200); max |ΔE| vs FP64 oracle"
+UNIT = "evals/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--engine", default="tc", choices=["simt", "tc", "paper"])
+    ap.add_argument("--warps", type=int, default=0, help="warps per CTA (0 = library choice)")
+    ap.add_argument("--config", type=int, default=2, choices=[2, 3])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-paper-engine", action="store_true")
+    return ap.parse_args()
+
+
+def workload_config(w, lig, engine, extra=None):
+    c = {
+        "workload": f"{w.name}: {lig.n_atoms} atoms, {lig.n_tors} torsions, {lig.n_pairs} intra pairs, "
+                    f"{w.grid.nx}^3 grid x {w.grid.spacing} A ({w.grid.n_maps} maps), {w.runs} runs x {w.pop} pop "
+                    f"x {w.iters} ADADELTA iterations per GPU",
+        "poses_per_gpu": w.n_poses, "iters": w.iters, "runs": w.runs, "pop": w.pop,
+        "engine": engine, "l2": "flushed between timed steps (256 MiB write, outside the timed events)",
+        "inputs": "seeded synthetic ligand/receptor grids (paper_conf_sc_solis_vasquezts25_b200/synth.py)",
+    }
+    if extra:
+        c.update(extra)
+    return c
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, smax, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax = max(smax, float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def load_traffic(engine, config):
+    """dram bytes per launch of the LS kernel from a committed ncu --set full summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(path))
+        k = d.get("ls_kernel", {}).get(f"config{config}_{engine}")
+        return None if k is None else float(k["dram_bytes_per_launch"])
+    except (OSError, ValueError, KeyError):
+        return None
+
+
+def run_reference(args):
+    """--impl reference: the FP64 oracle as it stands, on host cores, rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    from paper_conf_sc_solis_vasquezts25_b200 import synth
+    w = synth.make_config(args.config)
+    lig = w.ligands[0]
+    cores = len(os.sched_getaffinity(0))
+    n_sample = 8 * cores if args.config == 2 else 2 * cores
+    genes = w.genes[:n_sample]
+    for _ in range(args.warmup):
+        O.local_search(lig, w.grid, w.ff, genes[:cores], max_iters=w.iters, threads=cores)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        O.local_search(lig, w.grid, w.ff, genes, max_iters=w.iters, threads=cores)
+    dt = time.perf_counter() - t0
+    evals = args.steps * n_sample * w.iters
+    val = evals / dt
+    sample = f"{n_sample} poses x {w.iters} ADADELTA iterations of {w.name} per step (of {w.n_poses} poses)"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": workload_config(w, lig, "oracle", {"sample": sample}),
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_solis_vasquezts25_b200 import ad, dist as addist, report, synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+
+    w = synth.make_config(args.config, replica=rank)
+    lig = w.ligands[0]
+    stride = lig.n_genes
+    ctx = ad.Context(local)
+    ctx.upload_grid(w.grid)
+    lid = ctx.upload_ligand(lig, w.ff)
+    start = torch.from_numpy(w.genes).to(dev)
+    genes = start.clone()
+    n = w.n_poses
+    bestE = torch.empty(n, device=dev)
+    run_best = torch.empty(w.runs, 1 + stride, device=dev)
+    n_evals = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    engine = ad.ENGINES[args.engine]
+    wpc = args.warps if args.engine != "paper" else (args.warps or 64)
+
+    def step(ev=None):
+        genes.copy_(start)
+        if ev:
+            ev[0].record(stream)
+        ad.ad_local_search(ctx.h, lid, None, genes, bestE, run_best, n_evals, max_iters=w.iters,
+                           pop_per_run=w.pop, engine=engine, warps_per_cta=wpc)
+        if ev:
+            ev[1].record(stream)
+        if world > 1:
+            addist.gather_records(run_best)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ev_step = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    ev_kern = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    n_evals.zero_()
+    with ClockSampler(local) as clocks:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        for k in range(args.steps):
+            flush.fill_(float(k))  # L2 flush, outside the timed events
+            ev_step[k][0].record(stream)
+            step(ev_kern[k])
+            ev_step[k][1].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev_step]
+    kern_ms = [a.elapsed_time(b) for a, b in ev_kern]
+    total = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(total, op=dist.ReduceOp.MAX)
+    total_ms = float(total.item())
+    assert int(n_evals.item()) == args.steps * n * w.iters
+    evals_all = world * args.steps * n * w.iters
+    value = evals_all / (total_ms / 1e3)
+
+    # ---- end to end through the public API with HOST buffers (pinned) ----
+    h_genes = torch.from_numpy(w.genes).pin_memory()
+    h_bestE = torch.empty(n).pin_memory()
+    h_run = torch.empty(w.runs, 1 + stride).pin_memory()
+    e2e_ev = []
+    for k in range(max(2, args.steps)):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        flush.fill_(float(k))
+        a.record(stream)
+        genes.copy_(h_genes, non_blocking=True)
+        ad.ad_local_search(ctx.h, lid, None, genes, bestE, run_best, None, max_iters=w.iters, pop_per_run=w.pop,
+                           engine=engine, warps_per_cta=wpc)
+        h_bestE.copy_(bestE, non_blocking=True)
+        h_run.copy_(run_best, non_blocking=True)
+        b.record(stream)
+        e2e_ev.append((a, b))
+    torch.cuda.synchronize()
+    e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_ev) / len(e2e_ev)
+    e2e_t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_val = world * n * w.iters / (float(e2e_t.item()) / 1e3)
+
+    # ---- paper-style baseline engine, same workload (speedup denominator) ----
+    paper = None
+    if rank == 0 and not args.no_paper_engine and args.engine != "paper":
+        gp = start.clone()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=2, warps_per_cta=64)
+        gp.copy_(start)
+        flush.fill_(1.0)
+        a.record(stream)
+        ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=2, warps_per_cta=64)
+        b.record(stream)
+        torch.cuda.synchronize()
+        pms = a.elapsed_time(b)
+        paper = {"engine": "paper-style baseline (block per pose, 64 threads, 7 sequential block reductions)",
+                 "ms_per_step": pms, "evals_per_s": n * w.iters / (pms / 1e3),
+                 "speedup_of_this_engine": pms / (statistics.median(kern_ms)),
+                 "paper_target_speedup": 1.35}
+
+    # ---- roofline of the dominant kernel (LS kernel), FP32 ALU bound ----
+    work = report.ligand_work(lig)
+    kern_avg_s = statistics.mean(kern_ms) / 1e3
+    achieved = work["flops"] * n * w.iters / kern_avg_s / 1e12
+    ck = clocks.summary()
+    peak = report.fp32_peak_tflops(1965.0)
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": load_traffic(args.engine, args.config),
+                "peak_basis": "148 SMs x 128 FP32 lanes x 2 (FMA) x 1965 MHz max SM clock (DESIGN.md)",
+                "flops_per_eval": work["flops"], "mufu_per_eval": work["mufu"],
+                "mufu_frac": work["mufu"] * n * w.iters / kern_avg_s / (148 * 16 * 1965e6),
+                "l2_gather_gbs": work["l2_bytes"] * n * w.iters / kern_avg_s / 1e9,
+                "kernel_ms_avg": kern_avg_s * 1e3}
+
+    # ---- CPU baseline (the oracle as it stands) + max |dE| vs the oracle ----
+    cpu = None
+    max_dE = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        from oracle import oracle as O
+        cores = len(os.sched_getaffinity(0))
+        n_s = 4 * cores
+        t0 = time.perf_counter()
+        O.local_search(lig, w.grid, w.ff, w.genes[:n_s], max_iters=w.iters, threads=cores)
+        dt = time.perf_counter() - t0
+        cpu = {"value": n_s * w.iters / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"{n_s} poses x {w.iters} ADADELTA iterations of {w.name}"}
+        # energy parity on the first 512 start poses, same launch configuration
+        ns = 512
+        gs = start[:ns].contiguous()
+        Eg, Gg, _ = ctx.score(lid, gs, grad=True)
+        torch.cuda.synchronize()
+        Eo, Go, aux, ag = O.score(lig, w.grid, w.ff, w.genes[:ns], threads=cores)
+        dE = np.abs(Eg.cpu().numpy().astype(np.float64) - Eo)
+        scale = aux[:, O.AUX_ABS_E] + aux[:, O.AUX_SENS_E]
+        sane = scale < 500
+        max_dE = {"max_abs_dE": float(dE.max()), "median_abs_dE": float(np.median(dE)),
+                  "max_abs_dE_sane_poses": float(dE[sane].max()) if sane.any() else None,
+                  "n_sane_poses": int(sane.sum()),
+                  "frac_within_gate": float(np.mean(dE <= 1e-3 + 2.0 ** -20 * scale)),
+                  "gate": "|dE| <= 1e-3 + 2^-20 (A_E + S_E) (DESIGN.md Tolerances); sane = A_E + S_E < 500",
+                  "sample": f"first {ns} start poses of {w.name}, ad_score_poses vs FP64 oracle"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": workload_config(w, lig, args.engine, {"parallelism": f"runs sharded, {world} GPU(s), "
+                                                                          "NCCL all_gather of best poses"}),
+            "roofline": roofline, "cpu_baseline": cpu, "parity": max_dE,
+            "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h_genes.numel() * 4),
+                    "d2h_bytes_per_step": int((h_bestE.numel() + h_run.numel()) * 4)},
+            "clocks": ck, "gpu_launches": 2 * args.steps,
+            "paper_baseline_engine": paper,
+        }
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,219 @@
+/*
+ * ad.h — C ABI of libad: the B200 (sm_100a) ADADELTA energy+gradient hot path
+ * of AutoDock-GPU as described in Solis-Vasquez et al., "Architecting Tensor
+ * Core-Based Reductions for Irregular Molecular Docking Kernels" (IA3 @ SC'25).
+ *
+ * Citations: P:Ln = /root/reference/PAPER.md line n.  Readings Z-k / O-k are
+ * the ones listed in DESIGN.md (originally SURVEY.md §8(c)).
+ *
+ * Conventions (all entry points):
+ *   - Every function returns an ad_status (int32): AD_OK = 0, negative = error.
+ *     No C++ exception, abort or exit crosses the ABI.  ad_last_error() returns
+ *     a thread-local, human-readable message for the last failing call.
+ *   - Host pointers are read during the call and never retained.  Device
+ *     pointers (pose, output and trace buffers) are caller-owned; the library
+ *     only reads/writes them from kernels enqueued on `cuda_stream`.
+ *   - `cuda_stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Compute calls enqueue asynchronously and return; a kernel fault
+ *     surfaces as AD_ERR_CUDA on a later call or stream synchronisation.
+ *     Device-side argument errors (bad pose_ligand ids) surface as
+ *     AD_ERR_INVALID_ARG on the NEXT call on the same context.
+ *   - One context per device per host thread (no internal locking).
+ *   - Units: Angstrom, kcal/mol, elementary charge, degrees (Z11).
+ */
+#ifndef AD_H
+#define AD_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum ad_status {
+    AD_OK = 0,
+    AD_ERR_INVALID_ARG = -1, /* null/inconsistent argument, index out of range */
+    AD_ERR_LIMIT = -2,       /* size beyond the compile-time limits below */
+    AD_ERR_CUDA = -3,        /* CUDA runtime error (message in ad_last_error) */
+    AD_ERR_OOM = -4,         /* device allocation failed */
+    AD_ERR_STATE = -5        /* call order violated (e.g. no grids uploaded) */
+};
+
+enum ad_engine {
+    /* Warp-per-pose kernel, gene-space sums by a warp prefix scan over atoms
+     * in torsion-tree DFS order (FP32 shuffles, no block barrier). */
+    AD_ENGINE_SIMT = 0,
+    /* Same kernel, gene-space sums D = M_ext * W as error-corrected TF32
+     * tensor-core MMAs (mma.sync m16n8k8; hi/lo split of W, accumulation
+     * outside the tensor core in FP32 round-to-nearest: P:L186-199). */
+    AD_ENGINE_TC = 1,
+    /* Paper-style baseline: one thread block per pose, 7 sequential
+     * block-level sum reductions per gradient plus
+     * shared-memory atomics, all on FP32 SIMT cores.  The speedup denominator. */
+    AD_ENGINE_PAPER_BASELINE = 2
+};
+
+/* Compile-time limits (violations return AD_ERR_LIMIT). */
+#define AD_MAX_ATOMS 256   /* u8 atom indices in the pair schedule */
+#define AD_MAX_TORS 58     /* 6 + 58 = 64 genes; AD-GPU supports 57 */
+#define AD_MAX_TYPES 32
+#define AD_MAX_MAPS 34     /* n_type_maps + electrostatic + desolvation */
+#define AD_MAX_LIGANDS 65536
+
+typedef struct ad_context ad_context;
+typedef int32_t ad_ligand_id;
+
+/* Thread-local message of the last failing call ("" if none). */
+const char* ad_last_error(void);
+
+/* Library ABI version (increments on incompatible changes). */
+int32_t ad_version(void);
+
+/* Create a context bound to CUDA device `cuda_device`.  *out receives the
+ * handle (NULL on failure).  Errors: AD_ERR_INVALID_ARG (out NULL / bad
+ * device), AD_ERR_CUDA. */
+int32_t ad_context_create(int32_t cuda_device, ad_context** out);
+
+/* Release every device buffer of the context (grids, ligands).  Synchronises
+ * the device first.  NULL is accepted (no-op). */
+int32_t ad_context_destroy(ad_context* ctx);
+
+/* Receptor grid maps (D3; AutoGrid maps listed by
+ * protein.maps.fld).  Grid point (i,j,k) sits at origin + spacing*(i,j,k);
+ * maps are [n_maps][nz][ny][nx], x fastest.  Maps 0..n_maps-3 are per-atom-type
+ * affinity maps, n_maps-2 the electrostatic map (multiplied by the atom
+ * charge q), n_maps-1 the desolvation map (multiplied by |q|).  O-2, Z5, Z20. */
+typedef struct {
+    int32_t nx, ny, nz; /* grid points per axis (>= 2 each) */
+    int32_t n_maps;     /* 3..AD_MAX_MAPS */
+    float spacing;      /* A, > 0 */
+    float origin[3];    /* A, position of grid point (0,0,0) */
+} ad_grid_desc;
+
+/* Copy the maps into library-owned device memory, re-laid out for the
+ * kernels' gathers (x-pair records, elec/desolv interleaved).
+ * `maps` is a host pointer, or a device pointer if maps_on_device != 0.
+ * Replaces any previous grid of the context.  Enqueued on `cuda_stream`; the
+ * caller may reuse `maps` when the call returns for host maps (copied
+ * synchronously), or after the stream completes for device maps.
+ * Errors: AD_ERR_INVALID_ARG, AD_ERR_LIMIT, AD_ERR_OOM, AD_ERR_CUDA. */
+int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* desc, const float* maps, int32_t maps_on_device,
+                        void* cuda_stream);
+
+/* Scoring-function constants (O-2, O-3; AutoDock4.2 defaults in DESIGN.md). */
+typedef struct {
+    float smooth;        /* A, width of the flat band around r0 (delta = smooth/2), Z6 */
+    float cut_vdw;       /* A, vdW / H-bond cutoff (strict <), Z7 */
+    float cut_el;        /* A, electrostatics / desolvation cutoff (strict <), Z7 */
+    float el_rmin;       /* A, floor on r in the electrostatic term, Z8 */
+    float diel_A, diel_B, diel_k, diel_lambda; /* eps(r) = A + B / (1 + k exp(-lambda B r)) */
+    float coeff_el;      /* kcal/mol A / e^2 (332.06363 x FE_coeff_estat) */
+    float coeff_ds;      /* FE_coeff_desolv */
+    float qasp;          /* charge-dependent desolvation factor Q */
+    float sigma_ds;      /* A, desolvation Gaussian width */
+    float w_out;         /* kcal/mol per (grid unit)^2, out-of-grid restraint, Z4 */
+} ad_ff_params;
+
+/* Ligand (D4-D7).  All pointers are HOST pointers, read and copied
+ * during ad_upload_ligand.  The library renumbers atoms internally (torsion-
+ * tree DFS order) and builds its own pose chains and pair schedule; outputs are
+ * in gene space only, so the renumbering is invisible to callers. */
+typedef struct {
+    int32_t n_atoms;            /* 1..AD_MAX_ATOMS */
+    int32_t n_tors;             /* 0..AD_MAX_TORS */
+    int32_t n_pairs;            /* >= 0 */
+    int32_t n_types;            /* 1..AD_MAX_TYPES */
+    const float* ref_xyz;       /* [n_atoms][3] A, rotation centre at the origin (Z22) */
+    const int32_t* atom_map;    /* [n_atoms] type-map index 0..n_maps-3 */
+    const int32_t* atom_type;   /* [n_atoms] intra type 0..n_types-1 */
+    const float* charge;        /* [n_atoms] e */
+    const int32_t* tors_axis;   /* [n_tors][2] (a fixed side, c moving side), listed root -> leaf (Z13) */
+    const uint8_t* tors_moving; /* [n_tors][n_atoms] 0/1; moving sets must be nested or disjoint
+                                   (a rotatable-bond tree), a not in its own set, c in it */
+    const int32_t* pairs;       /* [n_pairs][2] intramolecular contributors, i != j (Z9) */
+    const float* tp_coef;       /* [n_types][n_types][5] cA, cB, r0, m, n with m == 12 and
+                                   n in {6, 10} (12-6 vdW / 12-10 H-bond, Z10) */
+    const float* type_S;        /* [n_types] desolvation solvation parameter S */
+    const float* type_V;        /* [n_types] desolvation volume V */
+    const ad_ff_params* ff;     /* scoring constants for this ligand */
+} ad_ligand_desc;
+
+/* Upload a ligand; *out receives its id (>= 0).  Requires a grid (atom_map
+ * must index a type map).  Errors: AD_ERR_INVALID_ARG (bad index, a not
+ * excluded from its moving set, non-laminar moving sets, i == j pair,
+ * unsupported exponents), AD_ERR_LIMIT, AD_ERR_STATE (no grid), AD_ERR_OOM. */
+int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* desc, ad_ligand_id* out);
+
+/* Free a ligand's device blob (synchronises the device). */
+int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig);
+
+/* One energy (+ gradient) evaluation per pose: PoseCalculation -> InterGradient
+ * -> IntraGradient -> gene-space sums (Alg 4; energy = inter + intra,
+ * O-5).  One warp per pose.
+ *   lig          ligand of every pose (if pose_ligand == NULL).
+ *   pose_ligand  device [n_poses] ligand ids, or NULL.  Shared memory is then
+ *                sized for the largest live ligand, and every aligned group of
+ *                poses sharing a CTA must use one ligand (groups of 1, 2, 4 or 8
+ *                poses; keep runs of one ligand a multiple of 8 poses long).
+ *   genes        device [n_poses][geno_stride] FP32, geno_stride >= 6 + n_tors:
+ *                translation (grid units), phi, theta, alpha, torsions (degrees).
+ *   energy       device [n_poses] FP32 out.
+ *   grad         device [n_poses][geno_stride] FP32 out (dE/dgene, padding
+ *                columns untouched), or NULL for energy only (NEXT-1).
+ *   aux          device [n_poses][8] FP32 out or NULL: E_inter, E_intra,
+ *                torque xyz (kcal/mol), sum of atom gradients xyz (kcal/mol/A).
+ * n_poses == 0 is a no-op.  Errors: AD_ERR_INVALID_ARG, AD_ERR_STATE,
+ * AD_ERR_CUDA. */
+int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses,
+                       const float* genes, int32_t geno_stride, float* energy, float* grad, float* aux,
+                       void* cuda_stream);
+
+/* ADADELTA local-search parameters (Alg 3; Zeiler [19] P:L406). */
+typedef struct {
+    int32_t max_iters;      /* evaluations per pose (default 300); >= 1 */
+    float rho, eps;         /* decay and conditioning constants (0.8, 0.01; Z14) */
+    int32_t pop_per_run;    /* poses per run for run_best; 0 = no run_best */
+    int32_t engine;         /* enum ad_engine */
+    int32_t warps_per_cta;  /* poses per CTA for SIMT/TC (0 = library choice);
+                               threads per block for PAPER_BASELINE (0 = 64) */
+    float* trace;           /* optional device [n_poses][max_iters][1 + 2*geno_stride]:
+                               per evaluation E, genes, gradient (Z19 shadowed parity) */
+} ad_ls_params;
+
+/* ADADELTA local search, one pose per warp (or per block for
+ * PAPER_BASELINE), max_iters evaluations each: evaluate (E, grad) of the
+ * current genotype, keep it if E < best (strict; earliest wins), update every
+ * gene (Z15, Z16: no angle wrapping).  On return (stream order):
+ *   genes        in: start genotypes; out: best genotype per pose.
+ *   best_energy  device [n_poses] FP32 best energy.
+ *   run_best     device [n_poses/pop_per_run][1 + geno_stride] FP32 or NULL:
+ *                per run the lowest best_energy (ties -> lowest pose index)
+ *                followed by that pose's genes (O-8).  Requires
+ *                n_poses % pop_per_run == 0.
+ *   n_evals      device int64 accumulator or NULL; += n_poses * max_iters.
+ * Errors: AD_ERR_INVALID_ARG, AD_ERR_STATE, AD_ERR_CUDA. */
+int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses,
+                        float* genes, int32_t geno_stride, float* best_energy, float* run_best, int64_t* n_evals,
+                        const ad_ls_params* params, void* cuda_stream);
+
+/* Reduction-engine microbenchmark (config 4; Eq 1-5): sum each of
+ * n_comp components over n_partials per block.
+ *   partials  device [n_blocks][n_partials][n_comp] FP32
+ *   out       device [n_blocks][n_comp] FP32
+ *   engine    AD_ENGINE_SIMT (warp transpose-butterfly + one smem exchange),
+ *             AD_ENGINE_TC (ones-vector TF32 MMA, hi/lo split, RN accumulation
+ *             outside the tensor core), AD_ENGINE_PAPER_BASELINE (n_comp
+ *             sequential block reductions with barriers).
+ * n_partials in {32, 64, ..., 1024} (multiple of 32), n_comp in 1..64. */
+int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
+                         const float* partials, float* out, void* cuda_stream);
+
+/* Device properties useful to callers: number of SMs and the shared memory
+ * footprint (bytes) the SIMT/TC kernel uses per pose for ligand `lig`. */
+int32_t ad_query(ad_context* ctx, ad_ligand_id lig, int32_t* n_sms, int32_t* smem_per_pose, int32_t* blob_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* AD_H */

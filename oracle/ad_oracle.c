@@ -78,7 +78,7 @@ typedef struct {
 } ado_ligand;
 
 /* aux[] layout written by ado_eval */
-enum { AUX_EINTER = 0, AUX_EINTRA = 1, AUX_ABS_E = 2, AUX_MARGIN_E = 3, AUX_MARGIN_G = 4, AUX_N = 5 };
+enum { AUX_EINTER = 0, AUX_EINTRA = 1, AUX_ABS_E = 2, AUX_MARGIN_E = 3, AUX_MARGIN_G = 4, AUX_SENS_E = 5, AUX_N = 6 };
 
 /* ------------------------------------------------------------------------ */
 static void cross(const double a[3], const double b[3], double out[3]) {
@@ -142,7 +142,7 @@ static double gv(const ado_grid* G, int m, int x, int y, int z) {
  * (A) to the nearest energy discontinuity (grid boundary) / gradient kink
  * (cell face).                                                               */
 static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, const double X[3], double grad[3],
-                         double* abs_e, double abs_g[3], double* margin_e, double* margin_g) {
+                         double* abs_e, double abs_g[3], double* abs_h, double* margin_e, double* margin_g) {
     const int n[3] = {G->nx, G->ny, G->nz};
     const double h = G->spacing;
     double u[3];
@@ -171,6 +171,7 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
             abs_g[k] = fabs(grad[k]);
         }
         *abs_e = fabs(E);
+        *abs_h = 2.0 * F->w_out / (h * h);
         return E;
     }
     int i0[3];
@@ -182,7 +183,7 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
     const int m_e = G->n_maps - 2, m_d = G->n_maps - 1;
     const double coef[3] = {1.0, q, fabs(q)};
     const int mm[3] = {map, m_e, m_d};
-    double E = 0.0, dEdu[3] = {0.0, 0.0, 0.0}, aE = 0.0, aG[3] = {0.0, 0.0, 0.0};
+    double E = 0.0, dEdu[3] = {0.0, 0.0, 0.0}, aE = 0.0, aG[3] = {0.0, 0.0, 0.0}, aV = 0.0;
     for (int cz = 0; cz < 2; cz++)
         for (int cy = 0; cy < 2; cy++)
             for (int cx = 0; cx < 2; cx++) {
@@ -198,6 +199,7 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
                     const double v = coef[t] * gv(G, mm[t], i0[0] + cx, i0[1] + cy, i0[2] + cz);
                     E += wgt * v;
                     aE += fabs(wgt * v);
+                    aV += fabs(v);
                     for (int k = 0; k < 3; k++) {
                         dEdu[k] += dw[k] * v;
                         aG[k] += fabs(dw[k] * v);
@@ -209,6 +211,7 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
         abs_g[k] = aG[k] / h;
     }
     *abs_e = aE;
+    *abs_h = aV / (h * h);
     return E;
 }
 
@@ -222,12 +225,12 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
  * desolvation if r < cut_el:
  *   E = c_ds [(S_i + Q|q_i|) V_j + (S_j + Q|q_j|) V_i] exp(-r^2 / (2 sigma^2)). */
 static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, double r, double* dEdr, double* abs_e,
-                         double* abs_d, double* margin_e, double* margin_g) {
+                         double* abs_d, double* abs_dd, double* margin_e, double* margin_g) {
     const int ti = L->atom_type[i], tj = L->atom_type[j];
     const float* tp = L->tp_coef + ((size_t)ti * L->n_types + tj) * 5;
     const double cA = tp[0], cB = tp[1], r0 = tp[2], m = tp[3], nn = tp[4];
     const double qi = L->charge[i], qj = L->charge[j];
-    double E = 0.0, D = 0.0, aE = 0.0, aD = 0.0;
+    double E = 0.0, D = 0.0, aE = 0.0, aD = 0.0, aDD = 0.0;
     const double delta = 0.5 * F->smooth;
     double me = fmin(fabs(r - F->cut_vdw), fabs(r - F->cut_el));
     double mg = fmin(fmin(fabs(r - (r0 - delta)), fabs(r - (r0 + delta))), fabs(r - F->el_rmin));
@@ -242,6 +245,7 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         D += da - db;
         aE += fabs(ea) + fabs(eb);
         aD += fabs(da) + fabs(db);
+        aDD += dsdr * (m * (m + 1.0) * fabs(cA) * pow(s, -m - 2.0) + nn * (nn + 1.0) * fabs(cB) * pow(s, -nn - 2.0));
     }
     if (r < F->cut_el) {
         const double lB = F->diel_lambda * F->diel_B;
@@ -256,6 +260,7 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         D += del;
         aE += fabs(eel);
         aD += fabs(del);
+        aDD += 2.0 * fabs(del) / re;
         const double Si = L->type_S[ti], Sj = L->type_S[tj], Vi = L->type_V[ti], Vj = L->type_V[tj];
         const double pref = F->coeff_ds * ((Si + F->qasp * fabs(qi)) * Vj + (Sj + F->qasp * fabs(qj)) * Vi);
         const double s2 = F->sigma_ds * F->sigma_ds;
@@ -265,10 +270,12 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         D += dds;
         aE += fabs(eds);
         aD += fabs(dds);
+        aDD += fabs(eds) * (r * r / (s2 * s2) + 1.0 / s2);
     }
     *dEdr = D;
     *abs_e = aE;
     *abs_d = aD;
+    *abs_dd = aDD;
     *margin_e = me;
     *margin_g = mg;
     return E;
@@ -317,8 +324,13 @@ static void jacobian(const ado_ligand* L, const ado_grid* G, const double* g, co
 }
 
 /* One pose: E (O-5: inter + intra), gene gradient grad[G] (may be NULL),
- * aux[AUX_N] (may be NULL), agrad[G] = per-gene sum over terms of |term's
- * contribution| (Z18 scale; may be NULL), X_out [N][3] (may be NULL). */
+ * aux[AUX_N] (may be NULL), agrad[G] (may be NULL), X_out [N][3] (may be NULL).
+ * Condition numbers for the Z18 tolerance:
+ *   aux[AUX_ABS_E]  = sum over every energy term of |term|
+ *   aux[AUX_SENS_E] = sum over terms of |d term / d coordinates| x |coordinates|
+ *                     (first-order sensitivity of E to relative rounding of X)
+ *   agrad[k]        = sum over terms of |dX/dg_k| . (|term gradient| +
+ *                     |d term gradient / dX| x |X|)                         */
 int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const double* g, double* E_out, double* grad,
              double* aux, double* agrad, double* X_out) {
     const int N = L->n_atoms, Gn = 6 + L->n_tors;
@@ -331,18 +343,22 @@ int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const doub
     double T[3];
     ado_pose(L, G, g, X, T);
     jacobian(L, G, g, X, T, J);
-    double Einter = 0.0, Eintra = 0.0, AE = 0.0, ME = 1e30, MG = 1e30;
+    double Einter = 0.0, Eintra = 0.0, AE = 0.0, ME = 1e30, MG = 1e30, SE = 0.0;
+    /* |J| row norms per atom and gene (for the condition numbers) */
     for (int i = 0; i < N; i++) {
-        double gr[3], agr[3], ae, me, mg;
-        Einter += inter_atom(G, F, L->atom_map[i], (double)L->charge[i], X + 3 * i, gr, &ae, agr, &me, &mg);
+        const double xn = sqrt(dot(X + 3 * i, X + 3 * i));
+        double gr[3], agr[3], ae, ah, me, mg;
+        Einter += inter_atom(G, F, L->atom_map[i], (double)L->charge[i], X + 3 * i, gr, &ae, agr, &ah, &me, &mg);
         AE += ae;
+        SE += (agr[0] + agr[1] + agr[2]) * xn;      /* first-order sensitivity to coordinate rounding */
         ME = fmin(ME, me);
         MG = fmin(MG, mg);
         for (int k = 0; k < 3; k++) { gi[3 * i + k] += gr[k]; ag[3 * i + k] += agr[k]; }
         if (acc)
             for (int q = 0; q < Gn; q++) {
                 const double* Jq = J + ((size_t)i * Gn + q) * 3;
-                acc[q] += fabs(Jq[0]) * agr[0] + fabs(Jq[1]) * agr[1] + fabs(Jq[2]) * agr[2];
+                const double jn = fabs(Jq[0]) + fabs(Jq[1]) + fabs(Jq[2]);
+                acc[q] += fabs(Jq[0]) * agr[0] + fabs(Jq[1]) * agr[1] + fabs(Jq[2]) * agr[2] + jn * ah * xn;
             }
     }
     for (int p = 0; p < L->n_pairs; p++) {
@@ -350,9 +366,11 @@ int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const doub
         double d[3];
         for (int k = 0; k < 3; k++) d[k] = X[3 * i + k] - X[3 * j + k];
         const double r = sqrt(dot(d, d));
-        double dEdr, ae, ad, me, mg;
-        Eintra += intra_pair(L, F, i, j, r, &dEdr, &ae, &ad, &me, &mg);
+        double dEdr, ae, ad, add, me, mg;
+        Eintra += intra_pair(L, F, i, j, r, &dEdr, &ae, &ad, &add, &me, &mg);
+        const double xl = sqrt(dot(X + 3 * i, X + 3 * i)) + sqrt(dot(X + 3 * j, X + 3 * j));
         AE += ae;
+        SE += ad * xl;
         ME = fmin(ME, me);
         MG = fmin(MG, mg);
         if (r > 0.0) {
@@ -363,10 +381,11 @@ int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const doub
             }
             if (acc) {
                 const double fa[3] = {fabs(ad * d[0] / r), fabs(ad * d[1] / r), fabs(ad * d[2] / r)};
+                const double h2 = (add + ad / r) * xl;   /* |dF/dX| x coordinate magnitude */
                 for (int q = 0; q < Gn; q++) {
                     const double* Ji = J + ((size_t)i * Gn + q) * 3;
                     const double* Jj = J + ((size_t)j * Gn + q) * 3;
-                    for (int k = 0; k < 3; k++) acc[q] += (fabs(Ji[k]) + fabs(Jj[k])) * fa[k];
+                    for (int k = 0; k < 3; k++) acc[q] += (fabs(Ji[k]) + fabs(Jj[k])) * (fa[k] + h2);
                 }
             }
         }
@@ -387,6 +406,7 @@ int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const doub
         aux[AUX_ABS_E] = AE;
         aux[AUX_MARGIN_E] = ME;
         aux[AUX_MARGIN_G] = MG;
+        aux[AUX_SENS_E] = SE;
     }
     if (agrad)
         for (int q = 0; q < Gn; q++) agrad[q] = acc[q];

@@ -17,7 +17,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = os.path.join(HERE, "ad_oracle.c")
 LIB = os.path.join(HERE, "libad_oracle.so")
 
-AUX_EINTER, AUX_EINTRA, AUX_ABS_E, AUX_MARGIN_E, AUX_MARGIN_G, AUX_N = range(6)
+AUX_EINTER, AUX_EINTRA, AUX_ABS_E, AUX_MARGIN_E, AUX_MARGIN_G, AUX_SENS_E, AUX_N = range(7)
 
 _lock = threading.Lock()
 _lib = None

@@ -1,0 +1,703 @@
+// ad_api.cu — host side of libad: the C ABI declared in include/ad.h.
+//
+// Upload-time preprocessing turns the paper's inputs (receptor maps, ligand
+// with rotation list and intramolecular contributor list) into
+// the device layouts of ad_internal.h:
+//   * grids  -> x-pair records (type maps) and interleaved elec/desolv records,
+//   * ligand -> torsion-tree DFS renumbering (every moving set contiguous),
+//               per-atom leaf->root torsion chains with reference-frame axes,
+//               a conflict-free pair schedule (rounds of 32, K gradient slots),
+//               per-pair desolvation prefactors, (cA, cB, r0, n) table.
+// Launches pick warps-per-CTA from the occupancy calculator.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "ad.h"
+#include "ad_internal.h"
+#include "ad_kernels.cuh"
+
+using namespace adk;
+
+namespace {
+
+thread_local std::string g_err;
+
+int32_t fail(int32_t code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CUDA_TRY(expr)                                                                          \
+    do {                                                                                        \
+        cudaError_t e_ = (expr);                                                                \
+        if (e_ != cudaSuccess) {                                                                \
+            return fail(e_ == cudaErrorMemoryAllocation ? AD_ERR_OOM : AD_ERR_CUDA, "%s: %s (%s:%d)", \
+                        #expr, cudaGetErrorString(e_), __FILE__, __LINE__);                    \
+        }                                                                                       \
+    } while (0)
+
+struct LigSlot {
+    unsigned char* d_blob = nullptr;
+    int32_t blob_bytes = 0;
+    int32_t scratch_bytes = 0;   // per warp (SIMT/TC)
+    int32_t block_scratch = 0;   // per block (baseline)
+    int32_t n_atoms = 0, n_tors = 0;
+    bool live = false;
+};
+
+}  // namespace
+
+struct ad_context {
+    int device = 0;
+    int n_sms = 0;
+    int max_smem_optin = 0;
+    int smem_per_sm = 0;
+    bool has_grid = false;
+    GridDev grid{};
+    int32_t grid_n_type = 0;
+    void* d_tmap = nullptr;
+    void* d_ed = nullptr;
+    std::vector<LigSlot> ligs;
+    LigDev* d_ligtab = nullptr;
+    int32_t ligtab_cap = 0;
+    int32_t* d_err = nullptr;
+    float* d_scratch_out = nullptr;  // placeholder energy buffer (unused outputs)
+};
+
+namespace {
+
+int32_t set_device(ad_context* ctx) {
+    CUDA_TRY(cudaSetDevice(ctx->device));
+    return AD_OK;
+}
+
+// surfaces device-side argument errors recorded by earlier kernels
+int32_t check_device_err(ad_context* ctx) {
+    int32_t h = 0;
+    CUDA_TRY(cudaMemcpy(&h, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (h) {
+        CUDA_TRY(cudaMemset(ctx->d_err, 0, sizeof(int32_t)));
+        return fail(AD_ERR_INVALID_ARG, "a previous kernel reported %s%s%s",
+                    (h & ERR_BAD_LIGAND) ? "[pose_ligand id out of range] " : "",
+                    (h & ERR_FOOTPRINT) ? "[ligand footprint larger than `lig`'s] " : "",
+                    (h & ERR_MIXED_CTA) ? "[pose_ligand not uniform within a CTA group]" : "");
+    }
+    return AD_OK;
+}
+
+int32_t sync_ligtab(ad_context* ctx) {
+    const int n = (int)ctx->ligs.size();
+    if (n > ctx->ligtab_cap) {
+        int cap = std::max(64, ctx->ligtab_cap * 2);
+        while (cap < n) cap *= 2;
+        LigDev* d = nullptr;
+        CUDA_TRY(cudaMalloc(&d, sizeof(LigDev) * cap));
+        if (ctx->d_ligtab) cudaFree(ctx->d_ligtab);
+        ctx->d_ligtab = d;
+        ctx->ligtab_cap = cap;
+    }
+    std::vector<LigDev> h(n);
+    for (int i = 0; i < n; ++i)
+        h[i] = LigDev{ctx->ligs[i].live ? ctx->ligs[i].d_blob : nullptr, ctx->ligs[i].blob_bytes,
+                      ctx->ligs[i].scratch_bytes};
+    if (n) CUDA_TRY(cudaMemcpy(ctx->d_ligtab, h.data(), sizeof(LigDev) * n, cudaMemcpyHostToDevice));
+    return AD_OK;
+}
+
+// ---------------------------------------------------------------- blob build
+struct BlobBuilder {
+    std::vector<unsigned char> buf;
+    int32_t put(const void* src, size_t bytes) {
+        const int32_t off = (int32_t)buf.size();
+        buf.resize(align16(off + (int32_t)bytes), 0);
+        if (bytes) memcpy(buf.data() + off, src, bytes);
+        return off;
+    }
+};
+
+struct Schedule {
+    int rounds = 0, slots = 1;
+    std::vector<uint32_t> rec;  // [rounds*32]
+    std::vector<float> dsv;     // [rounds*32]
+};
+
+// Greedy packing of pairs into rounds of 32 where each atom occurs at most K
+// times per round; occurrence k of atom a in a round targets gradient slot k.
+// Pairs are visited in a fixed pseudo-random order (consecutive pairs of the
+// input list share atoms and would saturate K early); K in 1..4 (shared memory
+// grows with K), the fewest rounds win, ties -> smaller K.
+Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
+                        const std::vector<int>& ptp, const std::vector<float>& pdsv) {
+    const int P = (int)pi.size();
+    const int target = (P + 31) / 32;
+    Schedule best;
+    best.rounds = 1 << 30;
+    std::vector<int> perm(P);
+    for (int q = 0; q < P; ++q) perm[q] = q;
+    uint64_t st = 0x9E3779B97F4A7C15ull;
+    for (int q = P - 1; q > 0; --q) {  // Fisher-Yates with a fixed xorshift stream
+        st ^= st << 13; st ^= st >> 7; st ^= st << 17;
+        std::swap(perm[q], perm[(int)(st % (uint64_t)(q + 1))]);
+    }
+    for (int K = 1; K <= 4; ++K) {
+        std::vector<int> rem = perm;
+        std::vector<std::vector<std::pair<int, uint32_t>>> rounds;
+        std::vector<int> cnt(n_atoms);
+        while (!rem.empty()) {
+            std::fill(cnt.begin(), cnt.end(), 0);
+            std::vector<std::pair<int, uint32_t>> rnd;
+            std::vector<int> rest;
+            for (int q : rem) {
+                const int i = pi[q], j = pj[q];
+                if ((int)rnd.size() < 32 && cnt[i] < K && cnt[j] < K) {
+                    const uint32_t r = (uint32_t)i | ((uint32_t)j << 8) | ((uint32_t)cnt[i] << 16) |
+                                       ((uint32_t)cnt[j] << 20) | ((uint32_t)ptp[q] << 24);
+                    cnt[i]++;
+                    cnt[j]++;
+                    rnd.push_back({q, r});
+                } else {
+                    rest.push_back(q);
+                }
+            }
+            rounds.push_back(std::move(rnd));
+            rem.swap(rest);
+        }
+        const int R = (int)rounds.size();
+        if (R < best.rounds) {
+            best.rounds = R;
+            best.slots = K;
+            best.rec.assign((size_t)R * 32, 0u);  // i == j == 0 -> empty slot
+            best.dsv.assign((size_t)R * 32, 0.f);
+            for (int r = 0; r < R; ++r)
+                for (size_t l = 0; l < rounds[r].size(); ++l) {
+                    best.rec[(size_t)r * 32 + l] = rounds[r][l].second;
+                    best.dsv[(size_t)r * 32 + l] = pdsv[rounds[r][l].first];
+                }
+        }
+        if (R <= target) break;
+    }
+    (void)target;
+    if (P == 0) {
+        best.rounds = 0;
+        best.slots = 1;
+    }
+    return best;
+}
+
+}  // namespace
+
+// =========================================================================== ABI
+extern "C" {
+
+const char* ad_last_error(void) { return g_err.c_str(); }
+
+int32_t ad_version(void) { return 1; }
+
+int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
+    if (!out) return fail(AD_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    int n = 0;
+    CUDA_TRY(cudaGetDeviceCount(&n));
+    if (cuda_device < 0 || cuda_device >= n) return fail(AD_ERR_INVALID_ARG, "device %d not in [0,%d)", cuda_device, n);
+    ad_context* ctx = new (std::nothrow) ad_context();
+    if (!ctx) return fail(AD_ERR_OOM, "host allocation failed");
+    ctx->device = cuda_device;
+    cudaError_t e = cudaSetDevice(cuda_device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->n_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+    if (e == cudaSuccess)
+        e = cudaDeviceGetAttribute(&ctx->max_smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, cuda_device);
+    if (e == cudaSuccess)
+        e = cudaDeviceGetAttribute(&ctx->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, cuda_device);
+    if (e == cudaSuccess) e = cudaMalloc(&ctx->d_err, sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaMemset(ctx->d_err, 0, sizeof(int32_t));
+    if (e != cudaSuccess) {
+        delete ctx;
+        return fail(AD_ERR_CUDA, "context init: %s", cudaGetErrorString(e));
+    }
+    *out = ctx;
+    return AD_OK;
+}
+
+int32_t ad_context_destroy(ad_context* ctx) {
+    if (!ctx) return AD_OK;
+    cudaSetDevice(ctx->device);
+    cudaDeviceSynchronize();
+    for (auto& l : ctx->ligs)
+        if (l.d_blob) cudaFree(l.d_blob);
+    if (ctx->d_tmap) cudaFree(ctx->d_tmap);
+    if (ctx->d_ed) cudaFree(ctx->d_ed);
+    if (ctx->d_ligtab) cudaFree(ctx->d_ligtab);
+    if (ctx->d_err) cudaFree(ctx->d_err);
+    delete ctx;
+    return AD_OK;
+}
+
+int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* d, const float* maps, int32_t maps_on_device,
+                        void* stream) {
+    if (!ctx || !d || !maps) return fail(AD_ERR_INVALID_ARG, "null argument");
+    if (d->nx < 2 || d->ny < 2 || d->nz < 2) return fail(AD_ERR_INVALID_ARG, "grid needs >= 2 points per axis");
+    if (d->n_maps < 3 || d->n_maps > AD_MAX_MAPS) return fail(AD_ERR_LIMIT, "n_maps %d not in [3,%d]", d->n_maps, AD_MAX_MAPS);
+    if (!(d->spacing > 0.f) || !std::isfinite(d->spacing)) return fail(AD_ERR_INVALID_ARG, "spacing must be > 0");
+    const size_t plane = (size_t)d->nx * d->ny, vol = plane * d->nz;
+    if (vol > (size_t)1 << 31) return fail(AD_ERR_LIMIT, "grid too large");
+    if (int32_t rc = set_device(ctx)) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    std::vector<float> h(vol * d->n_maps);
+    if (maps_on_device) {
+        CUDA_TRY(cudaMemcpyAsync(h.data(), maps, sizeof(float) * h.size(), cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(cudaStreamSynchronize(st));
+    } else {
+        memcpy(h.data(), maps, sizeof(float) * h.size());
+    }
+    const int nt = d->n_maps - 2;
+    std::vector<float2> tm(vol * nt);
+    std::vector<float4> ed(vol);
+    for (int m = 0; m < nt; ++m)
+        for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
+            for (int x = 0; x < d->nx; ++x) {
+                const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
+                tm[m * vol + i] = make_float2(h[m * vol + i], h[m * vol + i1]);
+            }
+    const float* E = h.data() + (size_t)nt * vol;
+    const float* D = h.data() + (size_t)(nt + 1) * vol;
+    for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
+        for (int x = 0; x < d->nx; ++x) {
+            const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
+            ed[i] = make_float4(E[i], E[i1], D[i], D[i1]);
+        }
+    if (ctx->d_tmap) { cudaFree(ctx->d_tmap); ctx->d_tmap = nullptr; }
+    if (ctx->d_ed) { cudaFree(ctx->d_ed); ctx->d_ed = nullptr; }
+    ctx->has_grid = false;
+    CUDA_TRY(cudaMalloc(&ctx->d_tmap, sizeof(float2) * tm.size()));
+    CUDA_TRY(cudaMalloc(&ctx->d_ed, sizeof(float4) * ed.size()));
+    CUDA_TRY(cudaMemcpy(ctx->d_tmap, tm.data(), sizeof(float2) * tm.size(), cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMemcpy(ctx->d_ed, ed.data(), sizeof(float4) * ed.size(), cudaMemcpyHostToDevice));
+    GridDev& g = ctx->grid;
+    g.tmap = (const float2*)ctx->d_tmap;
+    g.ed = (const float4*)ctx->d_ed;
+    g.nx = d->nx; g.ny = d->ny; g.nz = d->nz; g.n_type = nt;
+    g.ox = d->origin[0]; g.oy = d->origin[1]; g.oz = d->origin[2];
+    g.h = d->spacing;
+    g.inv_h = 1.0f / d->spacing;
+    ctx->grid_n_type = nt;
+    ctx->has_grid = true;
+    return AD_OK;
+}
+
+int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id* out) {
+    if (!ctx || !d || !out) return fail(AD_ERR_INVALID_ARG, "null argument");
+    *out = -1;
+    if (!ctx->has_grid) return fail(AD_ERR_STATE, "upload grids before ligands");
+    const int N = d->n_atoms, T = d->n_tors, P = d->n_pairs, nt = d->n_types;
+    if (N < 1 || N > AD_MAX_ATOMS) return fail(AD_ERR_LIMIT, "n_atoms %d not in [1,%d]", N, AD_MAX_ATOMS);
+    if (T < 0 || T > AD_MAX_TORS) return fail(AD_ERR_LIMIT, "n_tors %d not in [0,%d]", T, AD_MAX_TORS);
+    if (nt < 1 || nt > AD_MAX_TYPES) return fail(AD_ERR_LIMIT, "n_types %d not in [1,%d]", nt, AD_MAX_TYPES);
+    if (P < 0) return fail(AD_ERR_INVALID_ARG, "n_pairs < 0");
+    if (!d->ref_xyz || !d->atom_map || !d->atom_type || !d->charge || !d->tp_coef || !d->type_S || !d->type_V ||
+        !d->ff || (T && (!d->tors_axis || !d->tors_moving)) || (P && !d->pairs))
+        return fail(AD_ERR_INVALID_ARG, "null array in ligand descriptor");
+    if ((int64_t)ctx->ligs.size() >= AD_MAX_LIGANDS) return fail(AD_ERR_LIMIT, "too many ligands");
+    for (int a = 0; a < N; ++a) {
+        if (d->atom_map[a] < 0 || d->atom_map[a] >= ctx->grid_n_type)
+            return fail(AD_ERR_INVALID_ARG, "atom_map[%d]=%d not a type map", a, d->atom_map[a]);
+        if (d->atom_type[a] < 0 || d->atom_type[a] >= nt)
+            return fail(AD_ERR_INVALID_ARG, "atom_type[%d]=%d out of range", a, d->atom_type[a]);
+    }
+    // --- torsion tree from the moving sets (must be laminar, listed root -> leaf)
+    std::vector<std::vector<uint8_t>> M(T, std::vector<uint8_t>(N));
+    std::vector<int> msize(T, 0);
+    for (int b = 0; b < T; ++b) {
+        for (int a = 0; a < N; ++a) {
+            M[b][a] = d->tors_moving[(size_t)b * N + a] ? 1 : 0;
+            msize[b] += M[b][a];
+        }
+        const int a0 = d->tors_axis[2 * b], c0 = d->tors_axis[2 * b + 1];
+        if (a0 < 0 || a0 >= N || c0 < 0 || c0 >= N || a0 == c0)
+            return fail(AD_ERR_INVALID_ARG, "torsion %d axis atoms out of range", b);
+        if (M[b][a0] || !M[b][c0])
+            return fail(AD_ERR_INVALID_ARG, "torsion %d: need a not moving and c moving", b);
+    }
+    std::vector<int> parent(T, -1);
+    for (int b = 0; b < T; ++b) {
+        for (int b2 = 0; b2 < T; ++b2) {
+            if (b2 == b) continue;
+            int inter = 0;
+            for (int a = 0; a < N; ++a) inter += M[b][a] & M[b2][a];
+            const bool sub = inter == msize[b], sup = inter == msize[b2], dis = inter == 0;
+            if (!sub && !sup && !dis) return fail(AD_ERR_INVALID_ARG, "moving sets of torsions %d and %d overlap", b, b2);
+            if (sub && msize[b] == msize[b2]) return fail(AD_ERR_INVALID_ARG, "torsions %d and %d move the same atoms", b, b2);
+            if (sub && b2 > b) return fail(AD_ERR_INVALID_ARG, "torsion %d listed before its parent %d (need root->leaf)", b, b2);
+            // every other torsion moves both axis atoms of b or neither
+            const int a0 = d->tors_axis[2 * b], c0 = d->tors_axis[2 * b + 1];
+            if (M[b2][a0] != M[b2][c0])
+                return fail(AD_ERR_INVALID_ARG, "torsion %d moves only one axis atom of torsion %d", b2, b);
+            if (sub && (parent[b] < 0 || msize[b2] < msize[parent[b]])) parent[b] = b2;
+        }
+    }
+    // --- DFS order: root atoms, then each torsion subtree (children in index order)
+    std::vector<int> order;
+    order.reserve(N);
+    std::vector<int> lo(T), hi(T);
+    std::vector<std::vector<int>> kids(T + 1);  // kids[T] = top level
+    for (int b = 0; b < T; ++b) kids[parent[b] < 0 ? T : parent[b]].push_back(b);
+    std::vector<int> owner(N, -1);  // deepest torsion moving the atom
+    for (int a = 0; a < N; ++a) {
+        int best = -1;
+        for (int b = 0; b < T; ++b)
+            if (M[b][a] && (best < 0 || msize[b] < msize[best])) best = b;
+        owner[a] = best;
+    }
+    struct Frame { int node; size_t next; };
+    std::vector<Frame> stack;
+    for (int a = 0; a < N; ++a)
+        if (owner[a] < 0) order.push_back(a);
+    for (int top : kids[T]) {
+        stack.push_back({top, 0});
+        lo[top] = (int)order.size();
+        for (int a = 0; a < N; ++a)
+            if (owner[a] == top) order.push_back(a);
+        while (!stack.empty()) {
+            Frame& f = stack.back();
+            if (f.next < kids[f.node].size()) {
+                const int c = kids[f.node][f.next++];
+                lo[c] = (int)order.size();
+                for (int a = 0; a < N; ++a)
+                    if (owner[a] == c) order.push_back(a);
+                stack.push_back({c, 0});
+            } else {
+                hi[f.node] = (int)order.size();
+                stack.pop_back();
+            }
+        }
+    }
+    if ((int)order.size() != N) return fail(AD_ERR_INVALID_ARG, "internal: DFS order incomplete");
+    std::vector<int> newi(N);
+    for (int k = 0; k < N; ++k) newi[order[k]] = k;
+    for (int b = 0; b < T; ++b)
+        if (hi[b] - lo[b] != msize[b]) return fail(AD_ERR_INVALID_ARG, "internal: moving set %d not contiguous", b);
+
+    // --- per-type-pair table
+    std::vector<float4> tp((size_t)nt * nt);
+    for (int t = 0; t < nt * nt; ++t) {
+        const float* c = d->tp_coef + 5 * t;
+        if (c[3] != 12.f || (c[4] != 6.f && c[4] != 10.f))
+            return fail(AD_ERR_INVALID_ARG, "tp_coef entry %d: exponents (%g,%g) unsupported (need 12-6 or 12-10)", t,
+                        c[3], c[4]);
+        tp[t] = make_float4(c[0], c[1], c[2], c[4]);
+    }
+    const ad_ff_params& F = *d->ff;
+    // --- pairs (new numbering) with desolvation prefactors
+    std::vector<int> pi(P), pj(P), ptp(P);
+    std::vector<float> pd(P);
+    for (int q = 0; q < P; ++q) {
+        const int i = d->pairs[2 * q], j = d->pairs[2 * q + 1];
+        if (i < 0 || i >= N || j < 0 || j >= N || i == j) return fail(AD_ERR_INVALID_ARG, "pair %d = (%d,%d) invalid", q, i, j);
+        pi[q] = newi[i];
+        pj[q] = newi[j];
+        const int ti = d->atom_type[i], tj = d->atom_type[j];
+        ptp[q] = ti * nt + tj;
+        const double qi = std::fabs((double)d->charge[i]), qj = std::fabs((double)d->charge[j]);
+        pd[q] = (float)((double)F.coeff_ds * (((double)d->type_S[ti] + (double)F.qasp * qi) * (double)d->type_V[tj] +
+                                              ((double)d->type_S[tj] + (double)F.qasp * qj) * (double)d->type_V[ti]));
+    }
+    if (nt * nt > 256) return fail(AD_ERR_LIMIT, "n_types^2 > 256");
+    const Schedule sch = schedule_pairs(N, pi, pj, ptp, pd);
+
+    // --- atoms, chains, masks (new numbering)
+    std::vector<float4> atoms(N);
+    std::vector<int2> info(N);
+    std::vector<uint8_t> chain;
+    std::vector<uint2> mask(N);
+    for (int k = 0; k < N; ++k) {
+        const int a = order[k];
+        atoms[k] = make_float4(d->ref_xyz[3 * a], d->ref_xyz[3 * a + 1], d->ref_xyz[3 * a + 2], d->charge[a]);
+        std::vector<int> ch;
+        uint64_t m = 0;
+        for (int b = 0; b < T; ++b)
+            if (M[b][a]) { ch.push_back(b); m |= 1ull << b; }
+        std::sort(ch.begin(), ch.end(), [&](int x, int y) { return msize[x] < msize[y]; });  // leaf -> root
+        info[k] = make_int2(d->atom_map[a] | (d->atom_type[a] << 8) | ((int)ch.size() << 16), (int)chain.size());
+        for (int b : ch) chain.push_back((uint8_t)b);
+        mask[k] = make_uint2((uint32_t)m, (uint32_t)(m >> 32));
+    }
+    std::vector<float4> tors(2 * std::max(T, 1));
+    std::vector<int4> tinfo(std::max(T, 1));
+    for (int b = 0; b < T; ++b) {
+        const int a0 = d->tors_axis[2 * b], c0 = d->tors_axis[2 * b + 1];
+        const double P0[3] = {d->ref_xyz[3 * a0], d->ref_xyz[3 * a0 + 1], d->ref_xyz[3 * a0 + 2]};
+        double u[3] = {d->ref_xyz[3 * c0] - P0[0], d->ref_xyz[3 * c0 + 1] - P0[1], d->ref_xyz[3 * c0 + 2] - P0[2]};
+        const double nu = std::sqrt(u[0] * u[0] + u[1] * u[1] + u[2] * u[2]);
+        if (!(nu > 0)) return fail(AD_ERR_INVALID_ARG, "torsion %d has a zero-length axis", b);
+        tors[2 * b] = make_float4((float)P0[0], (float)P0[1], (float)P0[2], 0.f);
+        tors[2 * b + 1] = make_float4((float)(u[0] / nu), (float)(u[1] / nu), (float)(u[2] / nu), 0.f);
+        tinfo[b] = make_int4(newi[a0], newi[c0], lo[b], hi[b]);
+    }
+
+    LigHeader H{};
+    H.n_atoms = N; H.n_tors = T; H.n_pairs = P; H.n_types = nt;
+    H.n_rounds = sch.rounds; H.n_slots = sch.slots; H.n_chain = (int)chain.size();
+    H.n_pad = (N + 7) & ~7;
+    const double sig = F.sigma_ds;
+    H.ff[FF_DELTA] = 0.5f * F.smooth;
+    H.ff[FF_CUT_VDW] = F.cut_vdw;
+    H.ff[FF_CUT_EL] = F.cut_el;
+    H.ff[FF_EL_RMIN] = F.el_rmin;
+    H.ff[FF_DIEL_A] = F.diel_A;
+    H.ff[FF_DIEL_B] = F.diel_B;
+    H.ff[FF_DIEL_K] = F.diel_k;
+    H.ff[FF_DIEL_LB] = (float)((double)F.diel_lambda * (double)F.diel_B);
+    H.ff[FF_COEFF_EL] = F.coeff_el;
+    H.ff[FF_DS_EXP2] = (float)(-1.4426950408889634 / (2.0 * sig * sig));
+    H.ff[FF_INV_S2] = (float)(1.0 / (sig * sig));
+    H.ff[FF_W_OUT] = F.w_out;
+    BlobBuilder B;
+    B.put(&H, sizeof(H));
+    H.off_atoms = B.put(atoms.data(), sizeof(float4) * N);
+    H.off_info = B.put(info.data(), sizeof(int2) * N);
+    H.off_tors = B.put(tors.data(), sizeof(float4) * 2 * T);
+    H.off_tinfo = B.put(tinfo.data(), sizeof(int4) * T);
+    H.off_chain = B.put(chain.data(), chain.size());
+    H.off_mask = B.put(mask.data(), sizeof(uint2) * N);
+    H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
+    H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
+    H.off_tp = B.put(tp.data(), sizeof(float4) * tp.size());
+    H.blob_bytes = (int32_t)B.buf.size();
+    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots);
+    H.scratch_bytes = ws.bytes;
+    memcpy(B.buf.data(), &H, sizeof(H));
+
+    if (int32_t rc = set_device(ctx)) return rc;
+    LigSlot s;
+    s.blob_bytes = H.blob_bytes;
+    s.scratch_bytes = ws.bytes;
+    s.block_scratch = block_scratch_layout(N, T).bytes;
+    s.n_atoms = N;
+    s.n_tors = T;
+    CUDA_TRY(cudaMalloc(&s.d_blob, B.buf.size()));
+    CUDA_TRY(cudaMemcpy(s.d_blob, B.buf.data(), B.buf.size(), cudaMemcpyHostToDevice));
+    s.live = true;
+    ctx->ligs.push_back(s);
+    if (int32_t rc = sync_ligtab(ctx)) return rc;
+    *out = (ad_ligand_id)(ctx->ligs.size() - 1);
+    return AD_OK;
+}
+
+int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig) {
+    if (!ctx || lig < 0 || lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live)
+        return fail(AD_ERR_INVALID_ARG, "bad ligand id %d", lig);
+    if (int32_t rc = set_device(ctx)) return rc;
+    CUDA_TRY(cudaDeviceSynchronize());
+    cudaFree(ctx->ligs[lig].d_blob);
+    ctx->ligs[lig] = LigSlot{};
+    return sync_ligtab(ctx);
+}
+
+}  // extern "C"
+
+// --------------------------------------------------------------- launches
+namespace {
+
+typedef void (*WarpKernel)(const KParams);
+
+WarpKernel pick_warp_kernel(int engine, bool grad, bool ls) {
+    if (ls) return engine == AD_ENGINE_TC ? k_warp_engine<1, true, true> : k_warp_engine<0, true, true>;
+    if (!grad) return k_warp_engine<0, false, false>;
+    return engine == AD_ENGINE_TC ? k_warp_engine<1, true, false> : k_warp_engine<0, true, false>;
+}
+
+int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const void* genes, int32_t stride) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (!ctx->has_grid) return fail(AD_ERR_STATE, "no grid uploaded");
+    if (lig < 0 || lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live) return fail(AD_ERR_INVALID_ARG, "bad ligand id %d", lig);
+    if (n_poses < 0) return fail(AD_ERR_INVALID_ARG, "n_poses < 0");
+    if (n_poses > 0 && !genes) return fail(AD_ERR_INVALID_ARG, "genes is NULL");
+    if (stride < 6 + ctx->ligs[lig].n_tors) return fail(AD_ERR_INVALID_ARG, "geno_stride %d < 6 + n_tors", stride);
+    return AD_OK;
+}
+
+// Choose warps per CTA: the most resident warps per SM, ties -> fewer warps per CTA
+// (finer load balance across SMs).
+int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int req_warps, cudaStream_t st) {
+    if (p.pose_ligand) {  // any live ligand may be referenced: size for the largest footprint
+        for (const LigSlot& o : ctx->ligs)
+            if (o.live) {
+                L.blob_bytes = std::max(L.blob_bytes, o.blob_bytes);
+                L.scratch_bytes = std::max(L.scratch_bytes, o.scratch_bytes);
+            }
+    }
+    const int cand[4] = {1, 2, 4, 8};
+    int best_w = 0, best_active = -1;
+    size_t best_smem = 0;
+    for (int w : cand) {
+        if (req_warps > 0 && w != req_warps) continue;
+        const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
+        if (smem > (size_t)ctx->max_smem_optin) continue;
+        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        int blocks = 0;
+        CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, kern, w * 32, smem));
+        const int active = blocks * w;
+        if (active > best_active) {
+            best_active = active;
+            best_w = w;
+            best_smem = smem;
+        }
+    }
+    if (best_w == 0 || best_active <= 0)
+        return fail(AD_ERR_LIMIT, "ligand footprint (%d B blob + %d B/warp) does not fit shared memory", L.blob_bytes,
+                    L.scratch_bytes);
+    p.smem_blob = L.blob_bytes;
+    p.smem_scratch = L.scratch_bytes;
+    const int grid = (p.n_poses + best_w - 1) / best_w;
+    kern<<<grid, best_w * 32, best_smem, st>>>(p);
+    CUDA_TRY(cudaGetLastError());
+    return AD_OK;
+}
+
+KParams base_params(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses, int32_t stride) {
+    KParams p{};
+    p.grid = ctx->grid;
+    p.ligs = ctx->d_ligtab;
+    p.lig = lig;
+    p.pose_ligand = pose_ligand;
+    p.n_poses = n_poses;
+    p.stride = stride;
+    p.err = ctx->d_err;
+    p.n_ligs = (int32_t)ctx->ligs.size();
+    p.max_iters = 1;
+    return p;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses,
+                       const float* genes, int32_t geno_stride, float* energy, float* grad, float* aux,
+                       void* stream) {
+    if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
+    if (n_poses > 0 && !energy) return fail(AD_ERR_INVALID_ARG, "energy is NULL");
+    if (int32_t rc = set_device(ctx)) return rc;
+    if (int32_t rc = check_device_err(ctx)) return rc;
+    if (n_poses == 0) return AD_OK;
+    KParams p = base_params(ctx, lig, pose_ligand, n_poses, geno_stride);
+    p.genes = const_cast<float*>(genes);
+    p.energy = energy;
+    p.grad = grad;
+    p.aux = aux;
+    const bool want_grad = grad != nullptr || aux != nullptr;
+    return launch_warp(ctx, ctx->ligs[lig], pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false), p, 0,
+                       (cudaStream_t)stream);
+}
+
+int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses, float* genes,
+                        int32_t geno_stride, float* best_energy, float* run_best, int64_t* n_evals,
+                        const ad_ls_params* prm, void* stream) {
+    if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
+    if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
+    if (prm->max_iters < 1) return fail(AD_ERR_INVALID_ARG, "max_iters must be >= 1");
+    if (prm->engine < 0 || prm->engine > 2) return fail(AD_ERR_INVALID_ARG, "unknown engine %d", prm->engine);
+    if (!(prm->rho >= 0.f && prm->rho < 1.f) || !(prm->eps > 0.f)) return fail(AD_ERR_INVALID_ARG, "need 0 <= rho < 1, eps > 0");
+    if (n_poses > 0 && !best_energy) return fail(AD_ERR_INVALID_ARG, "best_energy is NULL");
+    if (run_best && (prm->pop_per_run <= 0 || n_poses % prm->pop_per_run))
+        return fail(AD_ERR_INVALID_ARG, "run_best needs pop_per_run > 0 dividing n_poses");
+    if (int32_t rc = set_device(ctx)) return rc;
+    if (int32_t rc = check_device_err(ctx)) return rc;
+    if (n_poses == 0) return AD_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    KParams p = base_params(ctx, lig, pose_ligand, n_poses, geno_stride);
+    p.genes = genes;
+    p.energy = best_energy;
+    p.trace = prm->trace;
+    p.n_evals = n_evals;
+    p.max_iters = prm->max_iters;
+    p.rho = prm->rho;
+    p.eps = prm->eps;
+    const LigSlot& L = ctx->ligs[lig];
+    if (prm->engine == AD_ENGINE_PAPER_BASELINE) {
+        int threads = prm->warps_per_cta > 0 ? prm->warps_per_cta : 64;
+        if (threads % 32 || threads < 32 || threads > 256) return fail(AD_ERR_INVALID_ARG, "baseline block size %d", threads);
+        if (6 + L.n_tors > threads) return fail(AD_ERR_INVALID_ARG, "baseline needs >= 6 + n_tors threads");
+        int32_t blob = L.blob_bytes, bscr = L.block_scratch;
+        if (pose_ligand)
+            for (const LigSlot& o : ctx->ligs)
+                if (o.live) { blob = std::max(blob, o.blob_bytes); bscr = std::max(bscr, o.block_scratch); }
+        const size_t smem = (size_t)blob + bscr;
+        if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "ligand too large for the baseline engine");
+        CUDA_TRY(cudaFuncSetAttribute(k_block_baseline, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        p.smem_blob = blob;
+        p.smem_scratch = bscr;
+        k_block_baseline<<<n_poses, threads, smem, st>>>(p);
+        CUDA_TRY(cudaGetLastError());
+    } else {
+        int w = prm->warps_per_cta;
+        if (w != 0 && w != 1 && w != 2 && w != 4 && w != 8) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d", w);
+        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st)) return rc;
+    }
+    if (run_best) {
+        const int runs = n_poses / prm->pop_per_run;
+        k_best_of_run<<<(runs + 3) / 4, 128, 0, st>>>(best_energy, genes, geno_stride, 6 + L.n_tors,
+                                                      prm->pop_per_run, runs, run_best);
+        CUDA_TRY(cudaGetLastError());
+    }
+    return AD_OK;
+}
+
+int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
+                         const float* partials, float* out, void* stream) {
+    if (!ctx || !partials || !out) return fail(AD_ERR_INVALID_ARG, "null argument");
+    if (n_blocks < 0) return fail(AD_ERR_INVALID_ARG, "n_blocks < 0");
+    if (n_partials < 32 || n_partials > 1024 || n_partials % 32) return fail(AD_ERR_INVALID_ARG, "n_partials %d", n_partials);
+    if (n_comp < 1 || n_comp > 64) return fail(AD_ERR_INVALID_ARG, "n_comp %d not in [1,64]", n_comp);
+    if (int32_t rc = set_device(ctx)) return rc;
+    if (n_blocks == 0) return AD_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const int nw = n_partials / 32;
+    if (engine == AD_ENGINE_SIMT) {
+        const int cmax = n_comp <= 8 ? 8 : n_comp <= 16 ? 16 : n_comp <= 32 ? 32 : 64;
+        const size_t smem = sizeof(float) * nw * cmax;
+        switch (cmax) {
+            case 8: k_reduce_simt<8><<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp); break;
+            case 16: k_reduce_simt<16><<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp); break;
+            case 32: k_reduce_simt<32><<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp); break;
+            default: k_reduce_simt<64><<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp); break;
+        }
+    } else if (engine == AD_ENGINE_TC) {
+        const int c8 = (n_comp + 7) & ~7;
+        const size_t smem = sizeof(float) * ((size_t)nw * 32 * c8 + (size_t)nw * c8);
+        if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "TC reduce staging too large");
+        CUDA_TRY(cudaFuncSetAttribute(k_reduce_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        k_reduce_tc<<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp);
+    } else if (engine == AD_ENGINE_PAPER_BASELINE) {
+        k_reduce_paper<<<n_blocks, n_partials, 0, st>>>(partials, out, n_comp);
+    } else {
+        return fail(AD_ERR_INVALID_ARG, "unknown engine %d", engine);
+    }
+    CUDA_TRY(cudaGetLastError());
+    return AD_OK;
+}
+
+int32_t ad_query(ad_context* ctx, ad_ligand_id lig, int32_t* n_sms, int32_t* smem_per_pose, int32_t* blob_bytes) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (n_sms) *n_sms = ctx->n_sms;
+    if (lig >= 0) {
+        if (lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live) return fail(AD_ERR_INVALID_ARG, "bad ligand id %d", lig);
+        if (smem_per_pose) *smem_per_pose = ctx->ligs[lig].scratch_bytes;
+        if (blob_bytes) *blob_bytes = ctx->ligs[lig].blob_bytes;
+    }
+    return AD_OK;
+}
+
+}  // extern "C"

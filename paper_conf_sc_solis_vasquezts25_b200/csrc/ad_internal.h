@@ -1,0 +1,148 @@
+// ad_internal.h — device-side data layout of libad (not part of the ABI).
+//
+// A ligand lives in ONE contiguous, 16-byte aligned blob that a CTA stages into
+// shared memory with a single TMA bulk copy (cp.async.bulk) and keeps for all
+// max_iters ADADELTA iterations.  Layout (offsets in LigHeader, bytes):
+//
+//   LigHeader                                   144 B
+//   atoms   float4 [N]      reference x,y,z (A, DFS order), charge q
+//   info    int2   [N]      {map | type<<8 | chain_len<<16, chain_start}
+//   tors    float4 [T][2]   reference-frame axis point P_b and unit axis u_b
+//   tinfo   int4   [T]      {a_b, c_b, lo_b, hi_b}: axis atoms and the moving set
+//                           M_b = [lo_b, hi_b) (contiguous thanks to DFS order)
+//   chain   u8     [Lrot]   per atom: the torsions moving it, leaf -> root
+//   mask    u32x2  [N]      per atom bitmask of torsions moving it (baseline engine)
+//   prec    u32    [R*32]   pair schedule: i | j<<8 | slot_i<<16 | slot_j<<20 | tp<<24
+//                           (i == j marks an empty slot).  Within one round of 32
+//                           every (slot, atom) target is distinct -> no atomics.
+//   pdsv    f32    [R*32]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
+//   tp      float4 [nt*nt]  cA, cB, r0, n  (m == 12)
+//
+// Per-warp scratch (after the blob, one slice per warp), see WarpScratch below.
+#pragma once
+#include <cstdint>
+
+namespace adk {
+
+constexpr int kLanes = 32;
+constexpr int kMaxGenes = 64;
+
+// indices into LigHdr::ff
+enum {
+    FF_DELTA = 0,     // smooth / 2
+    FF_CUT_VDW = 1,
+    FF_CUT_EL = 2,
+    FF_EL_RMIN = 3,
+    FF_DIEL_A = 4,
+    FF_DIEL_B = 5,
+    FF_DIEL_K = 6,
+    FF_DIEL_LB = 7,   // lambda * B
+    FF_COEFF_EL = 8,
+    FF_DS_EXP2 = 9,   // -log2(e) / (2 sigma^2)
+    FF_INV_S2 = 10,   // 1 / sigma^2
+    FF_W_OUT = 11,
+    FF_N = 16
+};
+
+struct alignas(16) LigHeader {
+    int32_t n_atoms, n_tors, n_pairs, n_types;        // 16
+    int32_t n_rounds, n_slots, n_chain, blob_bytes;   // 32
+    int32_t off_atoms, off_info, off_tors, off_tinfo; // 48
+    int32_t off_chain, off_mask, off_prec, off_pdsv;  // 64
+    int32_t off_tp, scratch_bytes, n_pad, reserved;   // 80
+    float ff[FF_N];                                   // 144
+};
+static_assert(sizeof(LigHeader) == 144, "header size");
+
+// Device table entry, one per uploaded ligand.
+struct LigDev {
+    const unsigned char* blob;
+    int32_t blob_bytes;
+    int32_t scratch_bytes;
+};
+
+// Grid in device memory, x-pair layout:
+//   tmap [n_type][nz][ny][nx] float2 (v[x], v[x+1])
+//   ed   [nz][ny][nx]         float4 (E[x], E[x+1], D[x], D[x+1])
+struct GridDev {
+    const float2* tmap;
+    const float4* ed;
+    int32_t nx, ny, nz, n_type;
+    float ox, oy, oz, h, inv_h;
+};
+
+// Per-warp scratch layout (offsets in bytes from the warp's slice; 16-aligned).
+struct WarpScratch {
+    int32_t x;      // float4 [Npad]        world coords + charge
+    int32_t g;      // float4 [K][Npad]     atom gradient accumulators (slot 0 seeded with inter)
+    int32_t w;      // float4 [Npad+1][2]   prefix sums (SIMT) / W staging (TC)
+    int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
+    int32_t trig;   // float2 [T]           cos, sin of torsion angles
+    int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
+    int32_t genes;  // float  [64]
+    int32_t bytes;
+};
+
+__host__ __device__ inline int32_t align16(int32_t v) { return (v + 15) & ~15; }
+
+__host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int32_t n_tors, int32_t n_slots) {
+    WarpScratch s;
+    const int32_t npad = (n_atoms + 7) & ~7;
+    const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
+    int32_t o = 0;
+    s.x = o;     o += 16 * npad;
+    s.g = o;     o += 16 * npad * n_slots;
+    s.w = o;     o += 32 * (npad + 1);
+    s.d = o;     o += align16(4 * 8 * mpad);
+    s.trig = o;  o += align16(8 * (n_tors > 0 ? n_tors : 1));
+    s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
+    s.genes = o; o += 4 * kMaxGenes;
+    s.bytes = o;
+    return s;
+}
+
+// Baseline engine (one block per pose) shared-memory layout after the blob.
+struct BlockScratch {
+    int32_t x, g, trig, tw, tacc, red, genes, bytes;
+};
+
+__host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, int32_t n_tors) {
+    BlockScratch s;
+    int32_t o = 0;
+    const int32_t t1 = n_tors > 0 ? n_tors : 1;
+    s.x = o;     o += 16 * n_atoms;
+    s.g = o;     o += 16 * n_atoms;
+    s.trig = o;  o += align16(8 * t1);
+    s.tw = o;    o += 32 * t1;
+    s.tacc = o;  o += align16(4 * t1);
+    s.red = o;   o += 4 * 16;
+    s.genes = o; o += 4 * kMaxGenes;
+    s.bytes = o;
+    return s;
+}
+
+struct KParams {
+    GridDev grid;
+    const LigDev* ligs;
+    int32_t lig;
+    const int32_t* pose_ligand;
+    int32_t n_poses;
+    int32_t stride;
+    float* genes;
+    float* energy;
+    float* grad;
+    float* aux;
+    float* trace;
+    int64_t* n_evals;
+    int32_t* err;
+    int32_t max_iters;
+    float rho, eps;
+    int32_t smem_blob;      // bytes reserved for the blob in shared memory
+    int32_t smem_scratch;   // bytes per warp (SIMT/TC) or per block (baseline)
+    int32_t n_ligs;
+};
+
+// device error bits
+enum { ERR_BAD_LIGAND = 1, ERR_FOOTPRINT = 2, ERR_MIXED_CTA = 4 };
+
+}  // namespace adk

@@ -1,0 +1,44 @@
+"""Multi-GPU plumbing: shard independent (ligand, run) units over ranks, gather best poses.
+
+Every LGA run is independent (Alg 1 coarse level), so the
+only inter-GPU step is the final gather of fixed-size best-pose records
+[energy, genes...].  Units are packed by LPT (longest processing
+time first) on a cost model of one run's ADADELTA work.
+"""
+from __future__ import annotations
+
+import heapq
+
+
+def unit_cost(n_atoms: int, n_tors: int, n_pairs: int, pop: int, iters: int) -> float:
+    """Relative cost of one run: pop * iters * (pair + atom + rotation work), SURVEY §8(e)."""
+    return float(pop) * iters * (75.0 * n_pairs + 200.0 * n_atoms + 30.0 * (n_atoms + 2 * n_tors) + 100.0)
+
+
+def lpt_shard(costs, n_ranks: int):
+    """Greedy LPT: assign units (by descending cost) to the least-loaded rank.
+    Returns per-rank lists of unit indices, each sorted ascending (deterministic)."""
+    if n_ranks < 1:
+        raise ValueError("n_ranks >= 1")
+    heap = [(0.0, r) for r in range(n_ranks)]
+    heapq.heapify(heap)
+    out = [[] for _ in range(n_ranks)]
+    for u in sorted(range(len(costs)), key=lambda k: (-costs[k], k)):
+        load, r = heapq.heappop(heap)
+        out[r].append(u)
+        heapq.heappush(heap, (load + costs[u], r))
+    return [sorted(x) for x in out]
+
+
+def gather_records(records, group=None):
+    """all_gather_into_tensor of equally shaped per-rank record tensors [n, width]
+    -> [world * n, width] (NCCL over NVLink on GPU, gloo on CPU)."""
+    import torch
+    import torch.distributed as dist
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
+        return records
+    ws = dist.get_world_size(group)
+    out = torch.empty((ws * records.shape[0],) + tuple(records.shape[1:]), dtype=records.dtype,
+                      device=records.device)
+    dist.all_gather_into_tensor(out, records.contiguous(), group=group)
+    return out

@@ -1,0 +1,290 @@
+"""GPU parity of the CUDA path (through the C ABI) against the FP64 oracle.
+
+Gates (tests/parity.py): energy |dE| <= 1e-3 +
+2^-20 (A_E + S_E); gradient ||dg|| <= 1e-4 max(||g||, 1e-2 ||A_grad||).
+Evaluations within 1e-4 A of a non-smooth point of the scoring function (grid
+cell face / boundary, smoothing-band edge, cutoff; aux margins from the oracle)
+may legitimately fall on the other side in FP32; they are counted, must stay
+rare (< 2 %), and are excluded from the gate.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from oracle import oracle as O  # noqa: E402
+from paper_conf_sc_solis_vasquezts25_b200 import synth  # noqa: E402
+from tests.parity import energy_gate, energy_scale, grad_gate  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+KINK = 1e-4
+
+
+@pytest.fixture(scope="module")
+def ad():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_solis_vasquezts25_b200 import ad as _ad
+    return _ad
+
+
+@pytest.fixture(scope="module")
+def ctx(ad):
+    c = ad.Context(0)
+    yield c
+    c.close()
+
+
+_uploaded = {}
+
+
+def _setup(ctx, w, key):
+    """Upload grid + ligands of workload w (grid replaced when the key changes)."""
+    if _uploaded.get("grid") != key:
+        ctx.upload_grid(w.grid)
+        _uploaded.clear()
+        _uploaded["grid"] = key
+    ids = []
+    for k, L in enumerate(w.ligands):
+        lk = (key, k)
+        if lk not in _uploaded:
+            _uploaded[lk] = ctx.upload_ligand(L, w.ff)
+        ids.append(_uploaded[lk])
+    return ids
+
+
+def check_scores(L, grid, ff, genes, E, G=None, label=""):
+    n = len(genes)
+    Eo, Go, aux, ag = O.score(L, grid, ff, genes)
+    kinkE = aux[:, O.AUX_MARGIN_E] < KINK
+    kinkG = aux[:, O.AUX_MARGIN_G] < KINK
+    okE = energy_gate(E, Eo, energy_scale(aux)) | kinkE
+    assert okE.all(), f"{label}: {np.sum(~okE)} energies outside the gate, e.g. {np.nonzero(~okE)[0][:5]}"
+    if G is not None:
+        Gn = L.n_genes
+        okG = grad_gate(G[:, :Gn], Go[:, :Gn], ag[:, :Gn]) | kinkG | kinkE
+        assert okG.all(), f"{label}: {np.sum(~okG)} gradients outside the gate, e.g. {np.nonzero(~okG)[0][:5]}"
+    assert (kinkE | kinkG).mean() < 0.02 or n < 50
+    return Eo, aux
+
+
+@pytest.mark.parametrize("which,n", [("cfg1", 256), ("cfg2", 512), ("cfg3", 192)])
+def test_score_poses_parity(ctx, which, n, request):
+    w = request.getfixturevalue(which)
+    (lid,) = _setup(ctx, w, which)
+    L = w.ligands[0]
+    g = torch.from_numpy(w.genes[:n]).cuda()
+    E, G, A = ctx.score(lid, g, grad=True, aux=True)
+    E0, _, _ = ctx.score(lid, g, grad=False)
+    torch.cuda.synchronize()
+    E, G, A, E0 = E.cpu().numpy(), G.cpu().numpy(), A.cpu().numpy(), E0.cpu().numpy()
+    Eo, aux = check_scores(L, w.grid, w.ff, w.genes[:n], E, G, which)
+    check_scores(L, w.grid, w.ff, w.genes[:n], E0, None, which + " energy-only")
+    # aux: inter / intra split and Gtrans / Grigidrot consistency with the gradient
+    sc = energy_scale(aux)
+    assert np.all(np.abs(A[:, 0] - aux[:, O.AUX_EINTER]) <= 1e-3 + 2.0 ** -20 * sc)
+    assert np.all(np.abs(A[:, 1] - aux[:, O.AUX_EINTRA]) <= 1e-3 + 2.0 ** -20 * sc)
+    h = w.grid.spacing
+    assert np.allclose(G[:, :3], h * A[:, 5:8], rtol=1e-5, atol=1e-5 * np.abs(G[:, :3]).max())
+    # dE/dalpha = (pi/180) u . tau
+    ph, th = np.radians(w.genes[:n, 3]), np.radians(w.genes[:n, 4])
+    u = np.stack([np.sin(th) * np.cos(ph), np.sin(th) * np.sin(ph), np.cos(th)], 1)
+    ga = np.radians(1.0) * np.sum(u * A[:, 2:5], 1)
+    assert np.allclose(G[:, 5], ga, rtol=1e-4, atol=1e-4 * (np.abs(ga).max() + 1))
+
+
+def _ls(ctx, lid, genes, engine, iters, **kw):
+    g = torch.from_numpy(genes).cuda()
+    nev = torch.zeros(1, dtype=torch.int64, device="cuda")
+    out = ctx.local_search(lid, g, max_iters=iters, engine=engine, trace=True, n_evals=nev, **kw)
+    torch.cuda.synchronize()
+    return (out["trace"].cpu().numpy(), out["best_energy"].cpu().numpy(), g.cpu().numpy(), int(nev.item()), out)
+
+
+@pytest.mark.parametrize("engine", ["simt", "tc", "paper"])
+@pytest.mark.parametrize("which,n,iters", [("cfg1", 32, 40), ("cfg2", 32, 60), ("cfg3", 8, 12)])
+def test_local_search_shadowed_parity(ctx, engine, which, n, iters, request):
+    """Z19 (i): every traced step (genes_k, E_k, grad_k) re-evaluated by the oracle;
+    each ADADELTA update re-applied in FP64 from the GPU's own gradient history."""
+    w = request.getfixturevalue(which)
+    (lid,) = _setup(ctx, w, which)
+    L = w.ligands[0]
+    Gn = L.n_genes
+    wpc = 64 if engine == "paper" else 0
+    tr, bE, best_genes, nev, _ = _ls(ctx, lid, w.genes[:n], engine, iters, warps_per_cta=wpc)
+    stride = w.genes.shape[1]
+    assert nev == n * iters
+    # best tracking: strict <, earliest wins; genes out = genes at that step
+    k = np.argmin(tr[:, :, 0], axis=1)
+    assert np.array_equal(bE, tr[np.arange(n), k, 0])
+    assert np.array_equal(best_genes[:, :Gn], tr[np.arange(n), k, 1:1 + Gn])
+    # step 0 evaluates the start genes exactly
+    assert np.array_equal(tr[:, 0, 1:1 + Gn], w.genes[:n, :Gn])
+    # per-step energy + gradient parity on a sample of steps
+    rng = np.random.default_rng(0)
+    sel = rng.choice(n * iters, size=min(n * iters, 160), replace=False)
+    flat = tr.reshape(n * iters, -1)
+    check_scores(L, w.grid, w.ff, flat[sel, 1:1 + stride], flat[sel, 0], flat[sel, 1 + stride:], f"{which} {engine}")
+    # ADADELTA updates (FP64 replay of the GPU's gradients)
+    for p in range(min(n, 8)):
+        eg2 = np.zeros(Gn)
+        ed2 = np.zeros(Gn)
+        for s in range(iters - 1):
+            x = tr[p, s, 1:1 + Gn].astype(np.float64)
+            eg2, ed2, xn = O.adadelta_step(tr[p, s, 1 + stride:1 + stride + Gn], eg2, ed2, x)
+            got = tr[p, s + 1, 1:1 + Gn].astype(np.float64)
+            tol = 1e-5 * np.abs(xn - x) + 2.0 ** -22 * np.abs(xn) + 1e-30
+            assert np.all(np.abs(got - xn) <= tol), (p, s)
+
+
+def test_run_best_and_determinism(ctx, cfg2):
+    (lid,) = _setup(ctx, cfg2, "cfg2")
+    n, pop = 600, 150
+    outs = []
+    for _ in range(2):
+        g = torch.from_numpy(cfg2.genes[:n]).cuda()
+        o = ctx.local_search(lid, g, max_iters=20, engine="tc", pop_per_run=pop)
+        torch.cuda.synchronize()
+        outs.append((o["best_energy"].cpu().numpy(), o["run_best"].cpu().numpy(), g.cpu().numpy()))
+    bE, rb, genes = outs[0]
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][2], outs[1][2]), "not deterministic"
+    for r in range(n // pop):
+        i = r * pop + int(np.argmin(bE[r * pop:(r + 1) * pop]))
+        assert rb[r, 0] == bE[i]
+        assert np.array_equal(rb[r, 1:], genes[i])
+    ref = O.best_of_run(bE.astype(np.float64), pop)
+    assert np.array_equal(ref, [r * pop + int(np.argmin(bE[r * pop:(r + 1) * pop])) for r in range(n // pop)])
+
+
+def test_engines_agree_on_first_steps(ctx, cfg2):
+    (lid,) = _setup(ctx, cfg2, "cfg2")
+    trs = {e: _ls(ctx, lid, cfg2.genes[:16], e, 3, warps_per_cta=(64 if e == "paper" else 0))[0]
+           for e in ("simt", "tc", "paper")}
+    for e in ("tc", "paper"):
+        d = np.abs(trs[e][:, 0, 0].astype(np.float64) - trs["simt"][:, 0, 0])
+        assert np.all(d <= 1e-5 * np.abs(trs["simt"][:, 0, 0]) + 1e-3)
+
+
+def test_full_size_sampled(ctx, cfg2):
+    """BASELINE config 2 at full size (3000 poses x 300 iterations) in the bench
+    launch configuration (TC engine, library-chosen CTA shape): properties on all
+    poses, oracle parity on sampled evaluations."""
+    (lid,) = _setup(ctx, cfg2, "cfg2")
+    L = cfg2.ligands[0]
+    Gn = L.n_genes
+    stride = cfg2.genes.shape[1]
+    tr, bE, best_genes, nev, _ = _ls(ctx, lid, cfg2.genes, "tc", 300, pop_per_run=150)
+    n = cfg2.n_poses
+    assert nev == n * 300
+    assert np.array_equal(bE, tr[:, :, 0].min(axis=1))
+    assert np.all(np.isfinite(bE))
+    rng = np.random.default_rng(1)
+    sel = rng.choice(n * 300, size=96, replace=False)
+    flat = tr.reshape(n * 300, -1)
+    check_scores(L, cfg2.grid, cfg2.ff, flat[sel, 1:1 + stride], flat[sel, 0], flat[sel, 1 + stride:], "cfg2 full")
+    # the search makes progress: best energy well below the start energy for most poses
+    assert np.mean(bE < tr[:, 0, 0]) > 0.9
+
+
+def test_edge_cases(ctx, ad):
+    from tests.util import hand_ligand
+    grid = synth.make_grid(77, 24, synth.TYPESETS[3], 100)
+    ff = synth.FFParams()
+    _uploaded.clear()
+    ctx.upload_grid(grid)
+    # rigid ligand (no torsions, no pairs) and a single atom
+    rigid = hand_ligand([[0, 0, 0], [1.5, 0, 0], [1.5, 1.5, 0]], types=[0, 1, 2], charges=[0.2, -0.3, 0.1],
+                        tp=np.tile(np.array([0, 0, 4, 12, 6], np.float32), (3, 3, 1)))
+    one = hand_ligand([[0, 0, 0]], types=[1], charges=[0.4], tp=np.tile(np.array([0, 0, 4, 12, 6], np.float32), (2, 2, 1)))
+    for L in (rigid, one):
+        lid = ctx.upload_ligand(L, ff)
+        genes = synth.make_genotypes(3, 40, 0, grid)
+        genes[0, :3] = [-5.0, 3.0, 4.0]           # out of the grid
+        genes[1, :3] = [40.0, 40.0, 40.0]
+        g = torch.from_numpy(genes).cuda()
+        E, G, _ = ctx.score(lid, g)
+        torch.cuda.synchronize()
+        check_scores(L, grid, ff, genes, E.cpu().numpy(), G.cpu().numpy(), "edge")
+        tr, bE, *_ = _ls(ctx, lid, genes, "simt", 5)
+        assert np.all(np.isfinite(bE))
+    # n_poses == 0 is a no-op
+    lid = ctx.upload_ligand(rigid, ff)
+    e = torch.empty(0, 6, device="cuda")
+    ad.ad_score_poses(ctx.h, lid, None, e, torch.empty(0, device="cuda"))
+    ad.ad_local_search(ctx.h, lid, None, e, torch.empty(0, device="cuda"))
+    # argument errors
+    with pytest.raises(ad.AdError) as ex:
+        ad.ad_score_poses(ctx.h, 10 ** 6, None, torch.zeros(4, 6, device="cuda"), torch.empty(4, device="cuda"))
+    assert ex.value.code == ad.AD_ERR_INVALID_ARG
+    with pytest.raises(ad.AdError):
+        ad.ad_score_poses(ctx.h, lid, None, torch.zeros(4, 5, device="cuda"), torch.empty(4, device="cuda"))
+    with pytest.raises(ad.AdError):
+        ctx.local_search(lid, torch.zeros(4, 6, device="cuda"), engine=7)
+    # out-of-range pose_ligand ids surface on the next call
+    pl = torch.tensor([lid, 9999, lid, lid], dtype=torch.int32, device="cuda")
+    ad.ad_score_poses(ctx.h, lid, pl, torch.zeros(4, 6, device="cuda"), torch.empty(4, device="cuda"))
+    torch.cuda.synchronize()
+    with pytest.raises(ad.AdError) as ex:
+        ad.ad_score_poses(ctx.h, lid, None, torch.zeros(4, 6, device="cuda"), torch.empty(4, device="cuda"))
+    assert ex.value.code == ad.AD_ERR_INVALID_ARG
+    _uploaded.clear()
+
+
+def test_large_ligand_limits(ctx):
+    """Biggest shapes: 58 torsions (64 genes) and 200 atoms."""
+    grid = synth.make_grid(78, 96, synth.TYPESETS[8], 3000)
+    ff = synth.FFParams()
+    _uploaded.clear()
+    ctx.upload_grid(grid)
+    for seed, n_at, n_t in ((1, 150, 58), (2, 200, 4)):
+        L = synth.make_ligand(seed, n_at, n_t, 8, chainlike=True)
+        lid = ctx.upload_ligand(L, ff)
+        genes = synth.make_genotypes(seed, 24, n_t, grid, frac=0.1)
+        g = torch.from_numpy(genes).cuda()
+        E, G, _ = ctx.score(lid, g)
+        torch.cuda.synchronize()
+        check_scores(L, grid, ff, genes, E.cpu().numpy(), G.cpu().numpy(), f"N={n_at} T={n_t}")
+    _uploaded.clear()
+
+
+def test_multi_ligand_pose_ligand(ctx, ad):
+    grid = synth.make_grid(79, 40, synth.TYPESETS[6], 800)
+    ff = synth.FFParams()
+    _uploaded.clear()
+    ctx.upload_grid(grid)
+    ligs = [synth.make_ligand(100 + k, n, t, 6) for k, (n, t) in enumerate(((30, 5), (18, 3), (36, 9)))]
+    ids = [ctx.upload_ligand(L, ff) for L in ligs]
+    big = max(range(3), key=lambda k: ligs[k].n_pairs)
+    per = 8
+    stride = 6 + max(L.n_tors for L in ligs)
+    genes = np.zeros((3 * per, stride), np.float32)
+    pl = np.repeat(np.array(ids, np.int32), per)
+    for k, L in enumerate(ligs):
+        genes[k * per:(k + 1) * per] = synth.make_genotypes(k, per, L.n_tors, grid, stride=stride, frac=0.3)
+    g = torch.from_numpy(genes).cuda()
+    E = torch.empty(3 * per, device="cuda")
+    Gd = torch.zeros(3 * per, stride, device="cuda")
+    ad.ad_score_poses(ctx.h, ids[big], torch.from_numpy(pl).cuda(), g, E, Gd)
+    torch.cuda.synchronize()
+    for k, L in enumerate(ligs):
+        s = slice(k * per, (k + 1) * per)
+        check_scores(L, grid, ff, genes[s], E.cpu().numpy()[s], Gd.cpu().numpy()[s], f"ligand {k}")
+    _uploaded.clear()
+
+
+@pytest.mark.parametrize("engine", ["simt", "tc", "paper"])
+def test_reduction_engines_accuracy(ctx, ad, engine):
+    """Config 4: |S - S_exact| <= (ceil(log2 P) + 2) 2^-24 sum|x| (O-7)."""
+    import math
+    for P in (128, 256, 512, 1024):
+        for Cc in (8, 16, 24, 32, 40):
+            for dist in ("uniform", "logmag"):
+                x = synth.make_reduction_partials(P * 7 + Cc, 64, P, Cc, dist)
+                xd = torch.from_numpy(x).cuda()
+                o = torch.empty(64, Cc, device="cuda")
+                ad.ad_reduce_blocks(ctx.h, ad.ENGINES[engine], xd, o)
+                torch.cuda.synchronize()
+                o = o.cpu().numpy().astype(np.float64)
+                ex = np.array([[math.fsum(x[b, :, c].astype(np.float64)) for c in range(Cc)] for b in range(64)])
+                bound = (math.ceil(math.log2(P)) + 2) * 2.0 ** -24 * np.abs(x.astype(np.float64)).sum(axis=1)
+                assert np.all(np.abs(o - ex) <= bound), (P, Cc, dist)
