@@ -13,7 +13,7 @@ HEADERS = ["ad_internal.h", "ad_kernels.cuh"]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
-    "-O3", "-lineinfo", "-std=c++17",
+    "-O3", "-lineinfo", "-std=c++17", "-ftz=true",
     "-Xcompiler", "-fPIC", "-shared",
 ]
 

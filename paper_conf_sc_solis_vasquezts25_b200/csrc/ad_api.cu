@@ -134,15 +134,81 @@ struct Schedule {
     std::vector<float> dsv;     // [rounds*32]
 };
 
-// Greedy packing of pairs into rounds of 32 where each atom occurs at most K
-// times per round; occurrence k of atom a in a round targets gradient slot k.
+// Swap the roles of i and j in a schedule record (the pair term is symmetric;
+// the type-pair index keeps the caller's (i, j) order).
+uint32_t swap_ij(uint32_t r) {
+    const uint32_t i = r & 0xff, j = (r >> 8) & 0xff, si = (r >> 16) & 0xf, sj = (r >> 20) & 0xf;
+    return j | (i << 8) | (sj << 16) | (si << 20) | (r & 0xff000000u);
+}
+
+// Place the (<= 64) pairs of one step into 8 groups of 8 consecutive entries
+// (= the quarter-warps of the two sub-steps, the unit in which a 128-bit shared
+// load/store is serviced).  Within a group the first atoms should have distinct
+// residues mod 8 and so should the second atoms: then every LDS.128/STS.128 of
+// the pair loop (X_i, X_j, both gradient read-modify-writes, whose addresses are
+// slot*npad + atom with npad % 8 == 0) is bank-conflict free.  Greedy, with the
+// i/j orientation as a free choice; leftovers fill empty places (then conflicts
+// are allowed).  Returns 64 entries, first == -1 marks an empty place.
+std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms) {
+    std::vector<std::pair<int, uint32_t>> out(kPairsPerStep, {-1, 0u});
+    std::vector<char> taken(pool.size(), 0);
+    int left = (int)pool.size();
+    const int groups = kPairsPerStep / 8;
+    // spread the load: about ceil(n/8) entries per group
+    const int per = (left + groups - 1) / groups;
+    for (int g = 0; g < groups && left; ++g) {
+        unsigned usedA = 0, usedB = 0;
+        int n = 0;
+        for (size_t e = 0; e < pool.size() && n < per; ++e) {
+            if (taken[e]) continue;
+            uint32_t r = pool[e].second;
+            unsigned a = r & 7u, b = (r >> 8) & 7u;
+            if ((usedA >> a & 1u) || (usedB >> b & 1u)) {
+                if ((usedA >> b & 1u) || (usedB >> a & 1u)) continue;
+                r = swap_ij(r);
+                std::swap(a, b);
+            }
+            usedA |= 1u << a;
+            usedB |= 1u << b;
+            out[g * 8 + n] = {pool[e].first, r};
+            taken[e] = 1;
+            ++n;
+            --left;
+        }
+    }
+    for (size_t e = 0, slot = 0; e < pool.size(); ++e) {  // leftovers: any empty place
+        if (taken[e]) continue;
+        while (out[slot].first >= 0) ++slot;
+        out[slot] = pool[e];
+    }
+    // empty places still issue their loads: point them (i == j == d marks an
+    // empty place) at an atom whose residue is unused in the group
+    for (int g = 0; g < groups; ++g) {
+        unsigned used = 0;
+        for (int k = 0; k < 8; ++k)
+            if (out[g * 8 + k].first >= 0) used |= (1u << (out[g * 8 + k].second & 7u)) | (1u << ((out[g * 8 + k].second >> 8) & 7u));
+        for (int k = 0; k < 8; ++k) {
+            if (out[g * 8 + k].first >= 0) continue;
+            unsigned d = 0;
+            while (d < 8 && d < (unsigned)n_atoms && (used >> d & 1u)) ++d;
+            if (d >= 8 || d >= (unsigned)n_atoms) d = 0;
+            used |= 1u << d;
+            out[g * 8 + k].second = d | (d << 8);
+        }
+    }
+    return out;
+}
+
+// Greedy packing of pairs into steps of 64 (2 per lane) where each atom occurs
+// at most K times per step; occurrence k of atom a in a step targets gradient
+// slot k, so all 128 read-modify-writes of a step hit distinct addresses.
 // Pairs are visited in a fixed pseudo-random order (consecutive pairs of the
 // input list share atoms and would saturate K early); K in 1..4 (shared memory
 // grows with K), the fewest rounds win, ties -> smaller K.
 Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
                         const std::vector<int>& ptp, const std::vector<float>& pdsv) {
     const int P = (int)pi.size();
-    const int target = (P + 31) / 32;
+    const int target = (P + kPairsPerStep - 1) / kPairsPerStep;
     Schedule best;
     best.rounds = 1 << 30;
     std::vector<int> perm(P);
@@ -152,7 +218,8 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         st ^= st << 13; st ^= st >> 7; st ^= st << 17;
         std::swap(perm[q], perm[(int)(st % (uint64_t)(q + 1))]);
     }
-    for (int K = 1; K <= 4; ++K) {
+    const int kmax = std::min(8, std::max(2, 256 / std::max(n_atoms, 1)));
+    for (int K = 1; K <= kmax; ++K) {
         std::vector<int> rem = perm;
         std::vector<std::vector<std::pair<int, uint32_t>>> rounds;
         std::vector<int> cnt(n_atoms);
@@ -162,7 +229,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
             std::vector<int> rest;
             for (int q : rem) {
                 const int i = pi[q], j = pj[q];
-                if ((int)rnd.size() < 32 && cnt[i] < K && cnt[j] < K) {
+                if ((int)rnd.size() < kPairsPerStep && cnt[i] < K && cnt[j] < K) {
                     const uint32_t r = (uint32_t)i | ((uint32_t)j << 8) | ((uint32_t)cnt[i] << 16) |
                                        ((uint32_t)cnt[j] << 20) | ((uint32_t)ptp[q] << 24);
                     cnt[i]++;
@@ -179,13 +246,16 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         if (R < best.rounds) {
             best.rounds = R;
             best.slots = K;
-            best.rec.assign((size_t)R * 32, 0u);  // i == j == 0 -> empty slot
-            best.dsv.assign((size_t)R * 32, 0.f);
-            for (int r = 0; r < R; ++r)
-                for (size_t l = 0; l < rounds[r].size(); ++l) {
-                    best.rec[(size_t)r * 32 + l] = rounds[r][l].second;
-                    best.dsv[(size_t)r * 32 + l] = pdsv[rounds[r][l].first];
+            best.rec.assign((size_t)R * kPairsPerStep, 0u);  // i == j == 0 -> empty slot
+            best.dsv.assign((size_t)R * kPairsPerStep, 0.f);
+            // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
+            for (int r = 0; r < R; ++r) {
+                const std::vector<std::pair<int, uint32_t>> lay = arrange_step(rounds[r], n_atoms);
+                for (int l = 0; l < kPairsPerStep; ++l) {
+                    best.rec[(size_t)r * kPairsPerStep + l] = lay[l].second;
+                    best.dsv[(size_t)r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
                 }
+            }
         }
         if (R <= target) break;
     }
@@ -473,7 +543,12 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.off_mask = B.put(mask.data(), sizeof(uint2) * N);
     H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
     H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
-    H.off_tp = B.put(tp.data(), sizeof(float4) * tp.size());
+    // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
+    // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
+    std::vector<float4> tp8(tp.size() * 8);
+    for (size_t t = 0; t < tp.size(); ++t)
+        for (int c = 0; c < 8; ++c) tp8[t * 8 + c] = tp[t];
+    H.off_tp = B.put(tp8.data(), sizeof(float4) * tp8.size());
     H.blob_bytes = (int32_t)B.buf.size();
     const WarpScratch ws = warp_scratch_layout(N, T, sch.slots);
     H.scratch_bytes = ws.bytes;
@@ -538,18 +613,25 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
                 L.scratch_bytes = std::max(L.scratch_bytes, o.scratch_bytes);
             }
     }
-    const int cand[4] = {1, 2, 4, 8};
-    int best_w = 0, best_active = -1;
+    // Every pose costs the same, so the launch is scored by (fewest waves of CTAs,
+    // then most resident warps per SM, then fewest warps per CTA).  Mixed-ligand
+    // launches keep power-of-two CTA sizes (pose_ligand groups must stay aligned).
+    int best_w = 0, best_active = -1, best_waves = 1 << 30;
     size_t best_smem = 0;
-    for (int w : cand) {
+    for (int w = 1; w <= 8; ++w) {
         if (req_warps > 0 && w != req_warps) continue;
+        if (p.pose_ligand && (w & (w - 1))) continue;
         const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
         if (smem > (size_t)ctx->max_smem_optin) continue;
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int blocks = 0;
         CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, kern, w * 32, smem));
+        if (blocks <= 0) continue;
         const int active = blocks * w;
-        if (active > best_active) {
+        const long ctas = (p.n_poses + w - 1) / w;
+        const int waves = (int)((ctas + (long)blocks * ctx->n_sms - 1) / ((long)blocks * ctx->n_sms));
+        if (waves < best_waves || (waves == best_waves && active > best_active)) {
+            best_waves = waves;
             best_active = active;
             best_w = w;
             best_smem = smem;
@@ -643,7 +725,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         CUDA_TRY(cudaGetLastError());
     } else {
         int w = prm->warps_per_cta;
-        if (w != 0 && w != 1 && w != 2 && w != 4 && w != 8) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d", w);
+        if (w < 0 || w > 8) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..8", w);
         if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st)) return rc;
     }
     if (run_best) {

@@ -12,11 +12,13 @@
 //                           M_b = [lo_b, hi_b) (contiguous thanks to DFS order)
 //   chain   u8     [Lrot]   per atom: the torsions moving it, leaf -> root
 //   mask    u32x2  [N]      per atom bitmask of torsions moving it (baseline engine)
-//   prec    u32    [R*32]   pair schedule: i | j<<8 | slot_i<<16 | slot_j<<20 | tp<<24
-//                           (i == j marks an empty slot).  Within one round of 32
-//                           every (slot, atom) target is distinct -> no atomics.
-//   pdsv    f32    [R*32]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
-//   tp      float4 [nt*nt]  cA, cB, r0, n  (m == 12)
+//   prec    u32    [R*64]   pair schedule: i | j<<8 | slot_i<<16 | slot_j<<20 | tp<<24
+//                           (i == j marks an empty slot).  Step r holds entries
+//                           [64r, 64r+64): lane l takes 64r+l and 64r+32+l; within a
+//                           step every (slot, atom) target is distinct -> no atomics.
+//   pdsv    f32    [R*64]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
+//   tp      float4 [nt*nt*8] cA, cB, r0, n (m == 12); 8 copies per entry (index t*8+c),
+//                           lane l reads copy l%8 -> conflict-free 128-bit lookups
 //
 // Per-warp scratch (after the blob, one slice per warp), see WarpScratch below.
 #pragma once
@@ -26,6 +28,7 @@ namespace adk {
 
 constexpr int kLanes = 32;
 constexpr int kMaxGenes = 64;
+constexpr int kPairsPerStep = 64;  // 2 pairs per lane per step of the intra loop
 
 // indices into LigHdr::ff
 enum {

@@ -58,13 +58,18 @@ def check_scores(L, grid, ff, genes, E, G=None, label=""):
     Eo, Go, aux, ag = O.score(L, grid, ff, genes)
     kinkE = aux[:, O.AUX_MARGIN_E] < KINK
     kinkG = aux[:, O.AUX_MARGIN_G] < KINK
-    okE = energy_gate(E, Eo, energy_scale(aux)) | kinkE
+    gE = energy_gate(E, Eo, energy_scale(aux))
+    okE = gE | kinkE
     assert okE.all(), f"{label}: {np.sum(~okE)} energies outside the gate, e.g. {np.nonzero(~okE)[0][:5]}"
+    excused = ~gE
     if G is not None:
         Gn = L.n_genes
-        okG = grad_gate(G[:, :Gn], Go[:, :Gn], ag[:, :Gn]) | kinkG | kinkE
+        gG = grad_gate(G[:, :Gn], Go[:, :Gn], ag[:, :Gn])
+        okG = gG | kinkG | kinkE
         assert okG.all(), f"{label}: {np.sum(~okG)} gradients outside the gate, e.g. {np.nonzero(~okG)[0][:5]}"
-    assert (kinkE | kinkG).mean() < 0.02 or n < 50
+        excused |= ~gG
+    # gate misses are only ever excused at a kink, and stay rare
+    assert excused.sum() <= max(1, int(0.02 * n)), f"{label}: {excused.sum()} kink-excused misses of {n}"
     return Eo, aux
 
 
