@@ -253,6 +253,7 @@ def main():
             dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev_step]
     kern_ms = [a.elapsed_time(b) for a, b in ev_kern]
+    launch = ad.ad_last_launch(ctx.h)
     total = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(total, op=dist.ReduceOp.MAX)
@@ -350,7 +351,9 @@ def main():
             "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": workload_config(w, lig, args.engine, {"parallelism": f"runs sharded, {world} GPU(s), "
-                                                                          "NCCL all_gather of best poses"}),
+                                                                          "NCCL all_gather of best poses",
+                                                            "launch": launch,
+                                                            "intra_mode": os.environ.get("AD_INTRA_MODE", "scatter")}),
             "roofline": roofline, "cpu_baseline": cpu, "parity": max_dE,
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h_genes.numel() * 4),
                     "d2h_bytes_per_step": int((h_bestE.numel() + h_run.numel()) * 4)},

@@ -212,6 +212,10 @@ int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int3
  * footprint (bytes) the SIMT/TC kernel uses per pose for ligand `lig`. */
 int32_t ad_query(ad_context* ctx, ad_ligand_id lig, int32_t* n_sms, int32_t* smem_per_pose, int32_t* blob_bytes);
 
+/* Launch shape of the last hot-path kernel enqueued on this context (for
+ * reporting): grid (CTAs), threads per CTA, dynamic shared memory bytes. */
+int32_t ad_last_launch(ad_context* ctx, int32_t* grid, int32_t* block, int32_t* smem_bytes);
+
 #ifdef __cplusplus
 }
 #endif

@@ -14,7 +14,7 @@ import threading
 import numpy as np
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libad.so")
+LIB_PATH = os.environ.get("AD_LIB", os.path.join(PKG, "libad.so"))  # AD_LIB: A/B builds
 
 AD_OK, AD_ERR_INVALID_ARG, AD_ERR_LIMIT, AD_ERR_CUDA, AD_ERR_OOM, AD_ERR_STATE = 0, -1, -2, -3, -4, -5
 AD_ENGINE_SIMT, AD_ENGINE_TC, AD_ENGINE_PAPER_BASELINE = 0, 1, 2
@@ -23,7 +23,7 @@ ENGINES = {"simt": AD_ENGINE_SIMT, "tc": AD_ENGINE_TC, "paper": AD_ENGINE_PAPER_
 # names exported by include/ad.h (tests check the .so exports all of them)
 EXPORTS = ("ad_last_error", "ad_version", "ad_context_create", "ad_context_destroy", "ad_upload_grids",
            "ad_upload_ligand", "ad_free_ligand", "ad_score_poses", "ad_local_search", "ad_reduce_blocks",
-           "ad_query")
+           "ad_query", "ad_last_launch")
 
 
 class AdError(RuntimeError):
@@ -79,6 +79,7 @@ def lib():
             L.ad_local_search.argtypes = [P, I32, P, I32, P, I32, P, P, P, C.POINTER(LSParams), P]
             L.ad_reduce_blocks.argtypes = [P, I32, I32, I32, I32, P, P, P]
             L.ad_query.argtypes = [P, I32, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
+            L.ad_last_launch.argtypes = [P, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
             for name in EXPORTS:
                 if name not in ("ad_last_error", "ad_version"):
                     getattr(L, name).restype = I32
@@ -188,6 +189,12 @@ def ad_query(ctx, lig=-1):
     a, b, c = C.c_int32(), C.c_int32(), C.c_int32()
     _check(lib().ad_query(ctx, lig, C.byref(a), C.byref(b), C.byref(c)))
     return {"n_sms": a.value, "smem_per_pose": b.value, "blob_bytes": c.value}
+
+
+def ad_last_launch(ctx):
+    a, b, c = C.c_int32(), C.c_int32(), C.c_int32()
+    _check(lib().ad_last_launch(ctx, C.byref(a), C.byref(b), C.byref(c)))
+    return {"grid": a.value, "block": b.value, "smem_bytes": c.value}
 
 
 # ---------------------------------------------------------------- convenience

@@ -74,7 +74,10 @@ struct ad_context {
     LigDev* d_ligtab = nullptr;
     int32_t ligtab_cap = 0;
     int32_t* d_err = nullptr;
-    float* d_scratch_out = nullptr;  // placeholder energy buffer (unused outputs)
+    // AD_INTRA_MODE=owner|scatter at context creation (tuning knob; scatter measured
+    // faster on config 2: 1.40e8 vs 1.26e8 evals/s, profiles/README.md)
+    int intra_mode = INTRA_SCATTER;
+    int32_t last_grid = 0, last_block = 0, last_smem = 0;
 };
 
 namespace {
@@ -149,7 +152,8 @@ uint32_t swap_ij(uint32_t r) {
 // slot*npad + atom with npad % 8 == 0) is bank-conflict free.  Greedy, with the
 // i/j orientation as a free choice; leftovers fill empty places (then conflicts
 // are allowed).  Returns 64 entries, first == -1 marks an empty place.
-std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms) {
+std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms,
+                                                   int K) {
     std::vector<std::pair<int, uint32_t>> out(kPairsPerStep, {-1, 0u});
     std::vector<char> taken(pool.size(), 0);
     int left = (int)pool.size();
@@ -193,7 +197,7 @@ std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<i
             while (d < 8 && d < (unsigned)n_atoms && (used >> d & 1u)) ++d;
             if (d >= 8 || d >= (unsigned)n_atoms) d = 0;
             used |= 1u << d;
-            out[g * 8 + k].second = d | (d << 8);
+            out[g * 8 + k].second = d | (d << 8) | ((uint32_t)K << 16) | ((uint32_t)K << 20);  // spare row K
         }
     }
     return out;
@@ -250,7 +254,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
             best.dsv.assign((size_t)R * kPairsPerStep, 0.f);
             // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
             for (int r = 0; r < R; ++r) {
-                const std::vector<std::pair<int, uint32_t>> lay = arrange_step(rounds[r], n_atoms);
+                const std::vector<std::pair<int, uint32_t>> lay = arrange_step(rounds[r], n_atoms, K);
                 for (int l = 0; l < kPairsPerStep; ++l) {
                     best.rec[(size_t)r * kPairsPerStep + l] = lay[l].second;
                     best.dsv[(size_t)r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
@@ -263,6 +267,188 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
     if (P == 0) {
         best.rounds = 0;
         best.slots = 1;
+    }
+    return best;
+}
+
+// Owner-computes list: every contributor pair (i, j) becomes two directed
+// entries (i <- j, primary) and (j <- i); entries are grouped by owner atom and
+// the concatenated list is cut into 32 equal slices (lane l takes entries
+// [l E, (l+1) E)), so every lane evaluates the same number of terms.  A lane
+// flushes its register accumulator whenever its owner atom changes: the k-th
+// flush of lane l goes to partial slot k*32 + l; comb/combidx list the slots of
+// every atom for the final per-atom sum.
+struct OwnerList {
+    int E = 0, C = 0;
+    std::vector<uint32_t> rec;  // [E][32]
+    std::vector<float> dsv;     // [E][32]
+    std::vector<int2> comb;     // [N]
+    std::vector<uint16_t> combidx;
+};
+
+OwnerList build_owner(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
+                      const std::vector<int>& ptp, const std::vector<float>& pdsv) {
+    struct Ent { int a, b, tp; float dsv; int primary; };
+    std::vector<std::vector<Ent>> lists(n_atoms);
+    for (size_t q = 0; q < pi.size(); ++q) {
+        lists[pi[q]].push_back({pi[q], pj[q], ptp[q], pdsv[q], 1});
+        lists[pj[q]].push_back({pj[q], pi[q], ptp[q], pdsv[q], 0});
+    }
+    std::vector<Ent> flat;
+    for (auto& l : lists) {
+        std::sort(l.begin(), l.end(), [](const Ent& x, const Ent& y) { return x.b < y.b; });
+        flat.insert(flat.end(), l.begin(), l.end());
+    }
+    OwnerList o;
+    const int total = (int)flat.size();
+    o.E = (total + 31) / 32;
+    o.rec.assign((size_t)o.E * 32, 0u);
+    o.dsv.assign((size_t)o.E * 32, 0.f);
+    std::vector<std::vector<uint16_t>> slots(n_atoms);
+    for (int l = 0; l < 32; ++l) {
+        int k = 0;
+        for (int t = 0; t < o.E; ++t) {
+            const int idx = l * o.E + t;
+            uint32_t fl;
+            int a = 0, b = 0, tp = 0;
+            float dv = 0.f;
+            if (idx < total) {
+                const Ent& e = flat[idx];
+                a = e.a; b = e.b; tp = e.tp; dv = e.dsv;
+                fl = e.primary ? OF_PRIMARY : 0;
+                if (t == 0 || flat[idx - 1].a != a) fl |= OF_FIRST;
+                if (t == o.E - 1 || idx == total - 1 || flat[idx + 1].a != a) {
+                    fl |= OF_LAST;
+                    slots[a].push_back((uint16_t)(k * 32 + l));
+                    ++k;
+                }
+            } else {
+                fl = OF_DUMMY | (t == 0 ? OF_FIRST : 0);
+            }
+            o.rec[(size_t)t * 32 + l] = (uint32_t)a | ((uint32_t)b << 8) | ((uint32_t)tp << 16) | (fl << 24);
+            o.dsv[(size_t)t * 32 + l] = dv;
+        }
+        o.C = std::max(o.C, k);
+    }
+    o.comb.resize(n_atoms);
+    for (int a = 0; a < n_atoms; ++a) {
+        o.comb[a] = make_int2((int)o.combidx.size(), (int)slots[a].size());
+        o.combidx.insert(o.combidx.end(), slots[a].begin(), slots[a].end());
+    }
+    return o;
+}
+
+// Hybrid list: every pair once, oriented owner i = min(i, j).  The owner-sorted
+// list is cut into 32 equal slices (one per lane); a lane walks its slice run by
+// run (a run = consecutive pairs with the same owner), keeps the owner's force in
+// registers and stores one partial per run (slot k*32 + lane, like the owner list).
+// The partner side is a read-modify-write of gradient slot s of atom j, with the
+// (slot, j) targets of the 64 pairs of a step distinct (no atomics, one
+// __syncwarp per step).  Steps are packed greedily per lane from its current run
+// (pairs of a run can be taken in any order); a lane with no fitting pair gets an
+// empty place (i == j == d, slot K = the spare row, flag OF_DUMMY).
+// Record: i | j<<8 | tp<<16 | slot<<24 (4 bits) | flags<<28 (OF_FIRST, OF_LAST, OF_DUMMY).
+struct HybridList {
+    int S = 0, K = 1, C = 0;
+    std::vector<uint32_t> rec;  // [S][2][32]
+    std::vector<float> dsv;
+    std::vector<int2> comb;
+    std::vector<uint16_t> combidx;
+};
+
+HybridList build_hybrid_k(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
+                          const std::vector<int>& ptp, const std::vector<float>& pdsv, int K) {
+    struct Pr { int i, j, tp; float dsv; };
+    std::vector<Pr> L;
+    for (size_t q = 0; q < pi.size(); ++q)
+        L.push_back({std::min(pi[q], pj[q]), std::max(pi[q], pj[q]), ptp[q], pdsv[q]});
+    std::sort(L.begin(), L.end(), [](const Pr& a, const Pr& b) { return a.i != b.i ? a.i < b.i : a.j < b.j; });
+    const int P = (int)L.size();
+    const int per = (P + 31) / 32;
+    // per lane: list of runs, each a vector of pairs
+    std::vector<std::vector<std::vector<Pr>>> runs(32);
+    for (int l = 0; l < 32; ++l)
+        for (int t = l * per; t < std::min(P, (l + 1) * per); ++t) {
+            if (runs[l].empty() || runs[l].back().front().i != L[t].i) runs[l].push_back({});
+            runs[l].back().push_back(L[t]);
+        }
+    struct LaneState { size_t run = 0; bool started = false; int flushes = 0; };
+    std::vector<LaneState> st(32);
+    HybridList h;
+    h.K = K;
+    std::vector<std::vector<uint16_t>> slots(n_atoms);
+    auto busy = [&](int l) { return st[l].run < runs[l].size(); };
+    std::vector<int> cnt(n_atoms);
+    while (true) {
+        bool any = false;
+        for (int l = 0; l < 32; ++l) any |= busy(l);
+        if (!any) break;
+        std::fill(cnt.begin(), cnt.end(), 0);
+        const size_t base = h.rec.size();
+        h.rec.resize(base + 64, 0u);
+        h.dsv.resize(base + 64, 0.f);
+        for (int u = 0; u < 2; ++u) {
+            unsigned used[4] = {0, 0, 0, 0};  // j residues per quarter-warp
+            for (int l = 0; l < 32; ++l) {
+                uint32_t rec = 0;
+                float dv = 0.f;
+                int pick = -1;
+                if (busy(l)) {
+                    std::vector<Pr>& run = runs[l][st[l].run];
+                    int fallback = -1;
+                    for (size_t c = 0; c < run.size(); ++c) {
+                        if (cnt[run[c].j] >= K) continue;
+                        if (!(used[l / 8] >> (run[c].j & 7) & 1u)) { pick = (int)c; break; }
+                        if (fallback < 0) fallback = (int)c;
+                    }
+                    if (pick < 0) pick = fallback;
+                    if (pick >= 0) {
+                        const Pr pr = run[pick];
+                        run.erase(run.begin() + pick);
+                        uint32_t fl = 0;
+                        if (!st[l].started) { fl |= OF_FIRST; st[l].started = true; }
+                        if (run.empty()) {
+                            fl |= OF_LAST;
+                            slots[pr.i].push_back((uint16_t)(st[l].flushes * 32 + l));
+                            st[l].flushes++;
+                            st[l].run++;
+                            st[l].started = false;
+                        }
+                        rec = (uint32_t)pr.i | ((uint32_t)pr.j << 8) | ((uint32_t)pr.tp << 16) |
+                              ((uint32_t)cnt[pr.j] << 24) | (fl << 28);
+                        cnt[pr.j]++;
+                        used[l / 8] |= 1u << (pr.j & 7);
+                        dv = pr.dsv;
+                    }
+                }
+                if (pick < 0) {  // empty place: spare row, a residue unused in the quarter if possible
+                    unsigned d = 0;
+                    while (d < 8 && d < (unsigned)n_atoms && (used[l / 8] >> d & 1u)) ++d;
+                    if (d >= 8 || d >= (unsigned)n_atoms) d = 0;
+                    used[l / 8] |= 1u << d;
+                    rec = d | (d << 8) | ((uint32_t)K << 24) | ((uint32_t)OF_DUMMY << 28);
+                }
+                h.rec[base + (size_t)u * 32 + l] = rec;
+                h.dsv[base + (size_t)u * 32 + l] = dv;
+            }
+        }
+        h.S++;
+    }
+    for (int l = 0; l < 32; ++l) h.C = std::max(h.C, st[l].flushes);
+    h.comb.resize(n_atoms);
+    for (int a = 0; a < n_atoms; ++a) {
+        h.comb[a] = make_int2((int)h.combidx.size(), (int)slots[a].size());
+        h.combidx.insert(h.combidx.end(), slots[a].begin(), slots[a].end());
+    }
+    return h;
+}
+
+HybridList build_hybrid(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
+                        const std::vector<int>& ptp, const std::vector<float>& pdsv) {
+    HybridList best;
+    for (int K = 1; K <= 4; ++K) {
+        HybridList h = build_hybrid_k(n_atoms, pi, pj, ptp, pdsv, K);
+        if (K == 1 || h.S < best.S) best = std::move(h);
     }
     return best;
 }
@@ -285,6 +471,8 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
     ad_context* ctx = new (std::nothrow) ad_context();
     if (!ctx) return fail(AD_ERR_OOM, "host allocation failed");
     ctx->device = cuda_device;
+    if (const char* m = getenv("AD_INTRA_MODE"))
+        ctx->intra_mode = strcmp(m, "owner") == 0 ? INTRA_OWNER : strcmp(m, "hybrid") == 0 ? INTRA_HYBRID : INTRA_SCATTER;
     cudaError_t e = cudaSetDevice(cuda_device);
     if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->n_sms, cudaDevAttrMultiProcessorCount, cuda_device);
     if (e == cudaSuccess)
@@ -484,7 +672,30 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
                                               ((double)d->type_S[tj] + (double)F.qasp * qj) * (double)d->type_V[ti]));
     }
     if (nt * nt > 256) return fail(AD_ERR_LIMIT, "n_types^2 > 256");
-    const Schedule sch = schedule_pairs(N, pi, pj, ptp, pd);
+    const int mode = ctx->intra_mode;
+    Schedule sch;
+    OwnerList own;
+    if (mode == INTRA_OWNER) {
+        own = build_owner(N, pi, pj, ptp, pd);
+        if (own.C * 32 > 65535) return fail(AD_ERR_LIMIT, "too many owner chunks");
+        sch.rounds = 0;
+        sch.slots = 1;
+        sch.rec = own.rec;
+        sch.dsv = own.dsv;
+    } else if (mode == INTRA_HYBRID) {
+        HybridList hy = build_hybrid(N, pi, pj, ptp, pd);
+        if (hy.C * 32 > 65535) return fail(AD_ERR_LIMIT, "too many hybrid runs");
+        sch.rounds = hy.S;
+        sch.slots = hy.K;
+        sch.rec = std::move(hy.rec);
+        sch.dsv = std::move(hy.dsv);
+        own.C = hy.C;
+        own.comb = std::move(hy.comb);
+        own.combidx = std::move(hy.combidx);
+    } else {
+        sch = schedule_pairs(N, pi, pj, ptp, pd);
+    }
+    if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
     // --- atoms, chains, masks (new numbering)
     std::vector<float4> atoms(N);
@@ -520,6 +731,9 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.n_atoms = N; H.n_tors = T; H.n_pairs = P; H.n_types = nt;
     H.n_rounds = sch.rounds; H.n_slots = sch.slots; H.n_chain = (int)chain.size();
     H.n_pad = (N + 7) & ~7;
+    H.intra_mode = mode;
+    H.n_entries = own.E;
+    H.n_chunks = own.C;
     const double sig = F.sigma_ds;
     H.ff[FF_DELTA] = 0.5f * F.smooth;
     H.ff[FF_CUT_VDW] = F.cut_vdw;
@@ -545,12 +759,14 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
     // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
     // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
-    std::vector<float4> tp8(tp.size() * 8);
+    std::vector<float4> tp8(tp.size() * AD_TP_COPIES);
     for (size_t t = 0; t < tp.size(); ++t)
-        for (int c = 0; c < 8; ++c) tp8[t * 8 + c] = tp[t];
+        for (int c = 0; c < AD_TP_COPIES; ++c) tp8[t * AD_TP_COPIES + c] = tp[t];
     H.off_tp = B.put(tp8.data(), sizeof(float4) * tp8.size());
+    H.off_comb = B.put(own.comb.data(), sizeof(int2) * own.comb.size());
+    H.off_combidx = B.put(own.combidx.data(), sizeof(uint16_t) * own.combidx.size());
     H.blob_bytes = (int32_t)B.buf.size();
-    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots);
+    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
     H.scratch_bytes = ws.bytes;
     memcpy(B.buf.data(), &H, sizeof(H));
 
@@ -630,6 +846,9 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
         const int active = blocks * w;
         const long ctas = (p.n_poses + w - 1) / w;
         const int waves = (int)((ctas + (long)blocks * ctx->n_sms - 1) / ((long)blocks * ctx->n_sms));
+        if (getenv("AD_DEBUG_LAUNCH"))
+            fprintf(stderr, "[libad] w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld waves=%d\n", w, smem, blocks,
+                    active, ctas, waves);
         if (waves < best_waves || (waves == best_waves && active > best_active)) {
             best_waves = waves;
             best_active = active;
@@ -644,6 +863,9 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     p.smem_scratch = L.scratch_bytes;
     const int grid = (p.n_poses + best_w - 1) / best_w;
     kern<<<grid, best_w * 32, best_smem, st>>>(p);
+    ctx->last_grid = grid;
+    ctx->last_block = best_w * 32;
+    ctx->last_smem = (int32_t)best_smem;
     CUDA_TRY(cudaGetLastError());
     return AD_OK;
 }
@@ -722,6 +944,9 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         p.smem_blob = blob;
         p.smem_scratch = bscr;
         k_block_baseline<<<n_poses, threads, smem, st>>>(p);
+        ctx->last_grid = n_poses;
+        ctx->last_block = threads;
+        ctx->last_smem = (int32_t)smem;
         CUDA_TRY(cudaGetLastError());
     } else {
         int w = prm->warps_per_cta;
@@ -768,6 +993,14 @@ int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int3
         return fail(AD_ERR_INVALID_ARG, "unknown engine %d", engine);
     }
     CUDA_TRY(cudaGetLastError());
+    return AD_OK;
+}
+
+int32_t ad_last_launch(ad_context* ctx, int32_t* grid, int32_t* block, int32_t* smem_bytes) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (grid) *grid = ctx->last_grid;
+    if (block) *block = ctx->last_block;
+    if (smem_bytes) *smem_bytes = ctx->last_smem;
     return AD_OK;
 }
 

@@ -17,6 +17,9 @@
 //                           [64r, 64r+64): lane l takes 64r+l and 64r+32+l; within a
 //                           step every (slot, atom) target is distinct -> no atomics.
 //   pdsv    f32    [R*64]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
+//           (INTRA_OWNER: prec/pdsv hold [E][32] directed entries a|b<<8|tp<<16|flags<<24
+//            instead, plus comb int2 [N] (start, count) into combidx u16 [..] = the
+//            partial slots k*32+lane that belong to atom a)
 //   tp      float4 [nt*nt*8] cA, cB, r0, n (m == 12); 8 copies per entry (index t*8+c),
 //                           lane l reads copy l%8 -> conflict-free 128-bit lookups
 //
@@ -47,15 +50,32 @@ enum {
     FF_N = 16
 };
 
+// Intra-pair evaluation modes (chosen at upload, uniform per ligand):
+//   INTRA_SCATTER: each pair evaluated once; steps of 64 pairs with distinct
+//                  (slot, atom) gradient targets -> read-modify-write, __syncwarp per step.
+//   INTRA_OWNER:   "owner computes": every pair evaluated from both ends (full
+//                  contributor list, 2x pair flops); lane l walks a balanced slice
+//                  of the atom-sorted directed list, accumulates g_a in registers and
+//                  stores one partial per (lane, atom chunk); no scatter, no sync in
+//                  the loop; partials are combined per atom afterwards.
+//   INTRA_HYBRID:  every pair once; the owner side (i = min(i, j)) accumulates in
+//                  registers along runs of equal owner, the partner side is a
+//                  conflict-free read-modify-write as in INTRA_SCATTER (half the
+//                  shared-memory RMW traffic, no duplicated flops).
+enum { INTRA_SCATTER = 0, INTRA_OWNER = 1, INTRA_HYBRID = 2 };
+// owner-mode entry: a | b<<8 | tp<<16 | flags<<24
+enum { OF_PRIMARY = 1, OF_FIRST = 2, OF_LAST = 4, OF_DUMMY = 8 };
+
 struct alignas(16) LigHeader {
-    int32_t n_atoms, n_tors, n_pairs, n_types;        // 16
-    int32_t n_rounds, n_slots, n_chain, blob_bytes;   // 32
-    int32_t off_atoms, off_info, off_tors, off_tinfo; // 48
-    int32_t off_chain, off_mask, off_prec, off_pdsv;  // 64
-    int32_t off_tp, scratch_bytes, n_pad, reserved;   // 80
-    float ff[FF_N];                                   // 144
+    int32_t n_atoms, n_tors, n_pairs, n_types;          // 16
+    int32_t n_rounds, n_slots, n_chain, blob_bytes;     // 32
+    int32_t off_atoms, off_info, off_tors, off_tinfo;   // 48
+    int32_t off_chain, off_mask, off_prec, off_pdsv;    // 64
+    int32_t off_tp, scratch_bytes, n_pad, intra_mode;   // 80
+    int32_t n_entries, n_chunks, off_comb, off_combidx; // 96  (owner mode: E per lane, chunks per lane)
+    float ff[FF_N];                                     // 160
 };
-static_assert(sizeof(LigHeader) == 144, "header size");
+static_assert(sizeof(LigHeader) == 160, "header size");
 
 // Device table entry, one per uploaded ligand.
 struct LigDev {
@@ -83,23 +103,26 @@ struct WarpScratch {
     int32_t trig;   // float2 [T]           cos, sin of torsion angles
     int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
     int32_t genes;  // float  [64]
+    int32_t part;   // float4 [C][32]       owner mode: per-(lane, chunk) partial gradients
     int32_t bytes;
 };
 
 __host__ __device__ inline int32_t align16(int32_t v) { return (v + 15) & ~15; }
 
-__host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int32_t n_tors, int32_t n_slots) {
+__host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int32_t n_tors, int32_t n_slots,
+                                                           int32_t n_chunks) {
     WarpScratch s;
     const int32_t npad = (n_atoms + 7) & ~7;
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
     int32_t o = 0;
     s.x = o;     o += 16 * npad;
-    s.g = o;     o += 16 * npad * n_slots;
+    s.g = o;     o += 16 * npad * (n_slots + 1);  // + spare row targeted by empty schedule places
     s.w = o;     o += 32 * (npad + 1);
     s.d = o;     o += align16(4 * 8 * mpad);
-    s.trig = o;  o += align16(8 * (n_tors > 0 ? n_tors : 1));
+    s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
     s.genes = o; o += 4 * kMaxGenes;
+    s.part = o;  o += 16 * 32 * n_chunks;
     s.bytes = o;
     return s;
 }
@@ -115,7 +138,7 @@ __host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, in
     const int32_t t1 = n_tors > 0 ? n_tors : 1;
     s.x = o;     o += 16 * n_atoms;
     s.g = o;     o += 16 * n_atoms;
-    s.trig = o;  o += align16(8 * t1);
+    s.trig = o;  o += align16(8 * (n_tors + 3));
     s.tw = o;    o += 32 * t1;
     s.tacc = o;  o += align16(4 * t1);
     s.red = o;   o += 4 * 16;
