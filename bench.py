@@ -40,7 +40,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--engine", default="tc", choices=["simt", "tc", "paper"])
+    # default = the faster engine measured on this workload (the TC engine is kept
+    # only if it wins, north_star); `--engine tc` times the tensor-core engine
+    ap.add_argument("--engine", default="simt", choices=["simt", "tc", "paper", "paper_tcec"])
     ap.add_argument("--warps", type=int, default=0, help="warps per CTA (0 = library choice)")
     ap.add_argument("--config", type=int, default=2, choices=[2, 3])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -218,7 +220,7 @@ def main():
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
     engine = ad.ENGINES[args.engine]
-    wpc = args.warps if args.engine != "paper" else (args.warps or 64)
+    wpc = args.warps if not args.engine.startswith("paper") else (args.warps or 64)
 
     def step(ev=None):
         genes.copy_(start)
@@ -287,21 +289,34 @@ def main():
 
     # ---- paper-style baseline engine, same workload (speedup denominator) ----
     paper = None
-    if rank == 0 and not args.no_paper_engine and args.engine != "paper":
-        gp = start.clone()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=2, warps_per_cta=64)
-        gp.copy_(start)
-        flush.fill_(1.0)
-        a.record(stream)
-        ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=2, warps_per_cta=64)
-        b.record(stream)
-        torch.cuda.synchronize()
-        pms = a.elapsed_time(b)
-        paper = {"engine": "paper-style baseline (block per pose, 64 threads, 7 sequential block reductions)",
-                 "ms_per_step": pms, "evals_per_s": n * w.iters / (pms / 1e3),
-                 "speedup_of_this_engine": pms / (statistics.median(kern_ms)),
-                 "paper_target_speedup": 1.35}
+    if rank == 0 and not args.no_paper_engine and not args.engine.startswith("paper"):
+        def time_engine(eng, threads):
+            gp = start.clone()
+            ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=eng,
+                               warps_per_cta=threads)
+            ts = []
+            for k in range(3):
+                gp.copy_(start)
+                flush.fill_(float(k))
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                ad.ad_local_search(ctx.h, lid, None, gp, bestE, None, None, max_iters=w.iters, engine=eng,
+                                   warps_per_cta=threads)
+                b.record(stream)
+                torch.cuda.synchronize()
+                ts.append(a.elapsed_time(b))
+            return statistics.median(ts)
+        base_ms = time_engine(ad.AD_ENGINE_PAPER_BASELINE, 64)
+        tcec_ms = time_engine(ad.AD_ENGINE_PAPER_TCEC, 64)
+        paper = {"engine": "paper-style kernel: block (64 threads) per pose, 7 sequential block reductions "
+                           "(SIMT baseline) or one error-corrected TF32 tensor-core reduction (TCEC)",
+                 "baseline_ms_per_step": base_ms, "tcec_ms_per_step": tcec_ms,
+                 "baseline_evals_per_s": n * w.iters / (base_ms / 1e3),
+                 "tcec_over_baseline": base_ms / tcec_ms,
+                 "speedup_of_this_engine": base_ms / (statistics.median(kern_ms)),
+                 "paper_target_speedup": 1.35,
+                 "paper_reported": "B200 TCEC/baseline 1.35x (42 cases, 256 threads, P:L299/L383); 1.45x 7cpa 128 "
+                                   "threads (Tab 5 P:L344)"}
 
     # ---- roofline of the dominant kernel (LS kernel), FP32 ALU bound ----
     work = report.ligand_work(lig)

@@ -50,7 +50,12 @@ enum ad_engine {
     /* Paper-style baseline: one thread block per pose, 7 sequential
      * block-level sum reductions per gradient plus
      * shared-memory atomics, all on FP32 SIMT cores.  The speedup denominator. */
-    AD_ENGINE_PAPER_BASELINE = 2
+    AD_ENGINE_PAPER_BASELINE = 2,
+    /* The same block-per-pose kernel with the seven reductions replaced by one
+     * tensor-core reduction of all seven values (ones-row MMA, Eq 1 generalised)
+     * with the TF32 hi/lo error correction: the paper's TCEC in its
+     * own design context (local search only). */
+    AD_ENGINE_PAPER_TCEC = 3
 };
 
 /* Compile-time limits (violations return AD_ERR_LIMIT). */

@@ -774,7 +774,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     LigSlot s;
     s.blob_bytes = H.blob_bytes;
     s.scratch_bytes = ws.bytes;
-    s.block_scratch = block_scratch_layout(N, T).bytes;
+    s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
     CUDA_TRY(cudaMalloc(&s.d_blob, B.buf.size()));
@@ -912,7 +912,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
     if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
     if (prm->max_iters < 1) return fail(AD_ERR_INVALID_ARG, "max_iters must be >= 1");
-    if (prm->engine < 0 || prm->engine > 2) return fail(AD_ERR_INVALID_ARG, "unknown engine %d", prm->engine);
+    if (prm->engine < 0 || prm->engine > 3) return fail(AD_ERR_INVALID_ARG, "unknown engine %d", prm->engine);
     if (!(prm->rho >= 0.f && prm->rho < 1.f) || !(prm->eps > 0.f)) return fail(AD_ERR_INVALID_ARG, "need 0 <= rho < 1, eps > 0");
     if (n_poses > 0 && !best_energy) return fail(AD_ERR_INVALID_ARG, "best_energy is NULL");
     if (run_best && (prm->pop_per_run <= 0 || n_poses % prm->pop_per_run))
@@ -930,20 +930,25 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     p.rho = prm->rho;
     p.eps = prm->eps;
     const LigSlot& L = ctx->ligs[lig];
-    if (prm->engine == AD_ENGINE_PAPER_BASELINE) {
+    if (prm->engine == AD_ENGINE_PAPER_BASELINE || prm->engine == AD_ENGINE_PAPER_TCEC) {
+        const bool tcec = prm->engine == AD_ENGINE_PAPER_TCEC;
         int threads = prm->warps_per_cta > 0 ? prm->warps_per_cta : 64;
         if (threads % 32 || threads < 32 || threads > 256) return fail(AD_ERR_INVALID_ARG, "baseline block size %d", threads);
         if (6 + L.n_tors > threads) return fail(AD_ERR_INVALID_ARG, "baseline needs >= 6 + n_tors threads");
-        int32_t blob = L.blob_bytes, bscr = L.block_scratch;
+        int32_t blob = L.blob_bytes, bscr = block_scratch_layout(L.n_atoms, L.n_tors, tcec ? threads : 0).bytes;
         if (pose_ligand)
             for (const LigSlot& o : ctx->ligs)
-                if (o.live) { blob = std::max(blob, o.blob_bytes); bscr = std::max(bscr, o.block_scratch); }
+                if (o.live) {
+                    blob = std::max(blob, o.blob_bytes);
+                    bscr = std::max(bscr, block_scratch_layout(o.n_atoms, o.n_tors, tcec ? threads : 0).bytes);
+                }
         const size_t smem = (size_t)blob + bscr;
         if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "ligand too large for the baseline engine");
-        CUDA_TRY(cudaFuncSetAttribute(k_block_baseline, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        void (*kern)(const KParams) = tcec ? k_block_baseline<true> : k_block_baseline<false>;
+        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         p.smem_blob = blob;
         p.smem_scratch = bscr;
-        k_block_baseline<<<n_poses, threads, smem, st>>>(p);
+        kern<<<n_poses, threads, smem, st>>>(p);
         ctx->last_grid = n_poses;
         ctx->last_block = threads;
         ctx->last_smem = (int32_t)smem;

@@ -129,10 +129,12 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
 
 // Baseline engine (one block per pose) shared-memory layout after the blob.
 struct BlockScratch {
-    int32_t x, g, trig, tw, tacc, red, genes, bytes;
+    int32_t x, g, trig, tw, tacc, red, genes, stage, bytes;
 };
 
-__host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, int32_t n_tors) {
+// stage: [stage_threads][8] floats for the TCEC variant's tensor-core reduction
+// (0 for the SIMT baseline, so its footprint is not inflated)
+__host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, int32_t n_tors, int32_t stage_threads) {
     BlockScratch s;
     int32_t o = 0;
     const int32_t t1 = n_tors > 0 ? n_tors : 1;
@@ -143,6 +145,7 @@ __host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, in
     s.tacc = o;  o += align16(4 * t1);
     s.red = o;   o += 4 * 16;
     s.genes = o; o += 4 * kMaxGenes;
+    s.stage = o; o += 32 * stage_threads;
     s.bytes = o;
     return s;
 }

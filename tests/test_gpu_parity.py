@@ -106,7 +106,7 @@ def _ls(ctx, lid, genes, engine, iters, **kw):
     return (out["trace"].cpu().numpy(), out["best_energy"].cpu().numpy(), g.cpu().numpy(), int(nev.item()), out)
 
 
-@pytest.mark.parametrize("engine", ["simt", "tc", "paper"])
+@pytest.mark.parametrize("engine", ["simt", "tc", "paper", "paper_tcec"])
 @pytest.mark.parametrize("which,n,iters", [("cfg1", 32, 40), ("cfg2", 32, 60), ("cfg3", 8, 12)])
 def test_local_search_shadowed_parity(ctx, engine, which, n, iters, request):
     """Z19 (i): every traced step (genes_k, E_k, grad_k) re-evaluated by the oracle;
@@ -115,7 +115,7 @@ def test_local_search_shadowed_parity(ctx, engine, which, n, iters, request):
     (lid,) = _setup(ctx, w, which)
     L = w.ligands[0]
     Gn = L.n_genes
-    wpc = 64 if engine == "paper" else 0
+    wpc = 64 if engine.startswith("paper") else 0
     tr, bE, best_genes, nev, _ = _ls(ctx, lid, w.genes[:n], engine, iters, warps_per_cta=wpc)
     stride = w.genes.shape[1]
     assert nev == n * iters
@@ -163,9 +163,9 @@ def test_run_best_and_determinism(ctx, cfg2):
 
 def test_engines_agree_on_first_steps(ctx, cfg2):
     (lid,) = _setup(ctx, cfg2, "cfg2")
-    trs = {e: _ls(ctx, lid, cfg2.genes[:16], e, 3, warps_per_cta=(64 if e == "paper" else 0))[0]
-           for e in ("simt", "tc", "paper")}
-    for e in ("tc", "paper"):
+    trs = {e: _ls(ctx, lid, cfg2.genes[:16], e, 3, warps_per_cta=(64 if e.startswith("paper") else 0))[0]
+           for e in ("simt", "tc", "paper", "paper_tcec")}
+    for e in ("tc", "paper", "paper_tcec"):
         d = np.abs(trs[e][:, 0, 0].astype(np.float64) - trs["simt"][:, 0, 0])
         assert np.all(d <= 1e-5 * np.abs(trs["simt"][:, 0, 0]) + 1e-3)
 

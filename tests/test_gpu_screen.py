@@ -1,0 +1,45 @@
+"""Config 5 (virtual screen) on one GPU: bucketed multi-ligand launches with
+pose_ligand must give exactly the per-ligand single launches' results (every
+pose's search is deterministic and independent of the CTA shape)."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from paper_conf_sc_solis_vasquezts25_b200 import synth  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+def test_screen_matches_single_ligand_runs():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_solis_vasquezts25_b200 import ad, screen
+    rng = np.random.default_rng(5)
+    grid = synth.make_grid(5100, 40, synth.TYPESETS[8], 800)
+    ff = synth.FFParams()
+    ligs = []
+    for k in range(12):
+        n = int(rng.integers(20, 70))
+        t = int(rng.integers(0, min(12, n // 3) + 1))
+        ligs.append(synth.make_ligand(777 + k, n, t, 8))
+    runs, pop, iters, stride = 2, 16, 20, 6 + 12
+    genes = np.concatenate([synth.make_genotypes(k, runs * pop, L.n_tors, grid, stride=stride, frac=0.3)
+                            for k, L in enumerate(ligs)])
+    ctx = ad.Context(0)
+    try:
+        rec, units = screen.run_screen(ctx, grid, ff, ligs, genes, runs, pop, iters, n_buckets=3)
+        rec = rec.cpu().numpy()
+        assert rec.shape[0] == len(units)
+        got = {(int(r[0]), int(r[1])): r[2:] for r in rec}
+        assert sorted(got) == sorted(units)
+        ctx.upload_grid(grid)
+        for k, L in enumerate(ligs):
+            lid = ctx.upload_ligand(L, ff)
+            g = torch.from_numpy(genes[k * runs * pop:(k + 1) * runs * pop].copy()).cuda()
+            out = ctx.local_search(lid, g, max_iters=iters, pop_per_run=pop)
+            rb = out["run_best"].cpu().numpy()
+            for r in range(runs):
+                assert np.array_equal(got[(k, r)], rb[r]), (k, r)
+    finally:
+        ctx.close()
