@@ -521,31 +521,64 @@ int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* d, const float* map
         memcpy(h.data(), maps, sizeof(float) * h.size());
     }
     const int nt = d->n_maps - 2;
-    std::vector<float2> tm(vol * nt);
-    std::vector<float4> ed(vol);
-    for (int m = 0; m < nt; ++m)
-        for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
-            for (int x = 0; x < d->nx; ++x) {
-                const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
-                tm[m * vol + i] = make_float2(h[m * vol + i], h[m * vol + i1]);
-            }
     const float* E = h.data() + (size_t)nt * vol;
     const float* D = h.data() + (size_t)(nt + 1) * vol;
-    for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
-        for (int x = 0; x < d->nx; ++x) {
-            const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
-            ed[i] = make_float4(E[i], E[i1], D[i], D[i1]);
-        }
+    // Cell records (3 x 256-bit loads per atom, 8x the map bytes) when they stay
+    // comfortably L2-resident, else x-pair records (8 loads per atom, 2x bytes).
+    const size_t cell_bytes = vol * ((size_t)nt * 32 + 64);
+    int layout = cell_bytes <= ((size_t)64 << 20) ? 1 : 0;
+    if (const char* e = getenv("AD_GRID_LAYOUT")) layout = strcmp(e, "cell") == 0 ? 1 : strcmp(e, "xpair") == 0 ? 0 : layout;
     if (ctx->d_tmap) { cudaFree(ctx->d_tmap); ctx->d_tmap = nullptr; }
     if (ctx->d_ed) { cudaFree(ctx->d_ed); ctx->d_ed = nullptr; }
     ctx->has_grid = false;
-    CUDA_TRY(cudaMalloc(&ctx->d_tmap, sizeof(float2) * tm.size()));
-    CUDA_TRY(cudaMalloc(&ctx->d_ed, sizeof(float4) * ed.size()));
-    CUDA_TRY(cudaMemcpy(ctx->d_tmap, tm.data(), sizeof(float2) * tm.size(), cudaMemcpyHostToDevice));
-    CUDA_TRY(cudaMemcpy(ctx->d_ed, ed.data(), sizeof(float4) * ed.size(), cudaMemcpyHostToDevice));
     GridDev& g = ctx->grid;
-    g.tmap = (const float2*)ctx->d_tmap;
-    g.ed = (const float4*)ctx->d_ed;
+    g = GridDev{};
+    if (layout == 1) {
+        auto at = [&](const float* m, int x, int y, int z) {
+            x = std::min(x, d->nx - 1); y = std::min(y, d->ny - 1); z = std::min(z, d->nz - 1);
+            return m[((size_t)z * d->ny + y) * d->nx + x];
+        };
+        std::vector<float> tc((size_t)nt * vol * 8), edc(vol * 16);
+        for (int z = 0; z < d->nz; ++z)
+            for (int y = 0; y < d->ny; ++y)
+                for (int x = 0; x < d->nx; ++x) {
+                    const size_t cell = ((size_t)z * d->ny + y) * d->nx + x;
+                    for (int c = 0; c < 8; ++c) {
+                        const int dx = c & 1, dy = (c >> 1) & 1, dz = c >> 2;
+                        for (int m = 0; m < nt; ++m)
+                            tc[((size_t)m * vol + cell) * 8 + c] = at(h.data() + (size_t)m * vol, x + dx, y + dy, z + dz);
+                        edc[cell * 16 + c] = at(E, x + dx, y + dy, z + dz);
+                        edc[cell * 16 + 8 + c] = at(D, x + dx, y + dy, z + dz);
+                    }
+                }
+        CUDA_TRY(cudaMalloc(&ctx->d_tmap, sizeof(float) * tc.size()));
+        CUDA_TRY(cudaMalloc(&ctx->d_ed, sizeof(float) * edc.size()));
+        CUDA_TRY(cudaMemcpy(ctx->d_tmap, tc.data(), sizeof(float) * tc.size(), cudaMemcpyHostToDevice));
+        CUDA_TRY(cudaMemcpy(ctx->d_ed, edc.data(), sizeof(float) * edc.size(), cudaMemcpyHostToDevice));
+        g.tc8 = (const float*)ctx->d_tmap;
+        g.ed8 = (const float*)ctx->d_ed;
+    } else {
+        std::vector<float2> tm(vol * nt);
+        std::vector<float4> ed(vol);
+        for (int m = 0; m < nt; ++m)
+            for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
+                for (int x = 0; x < d->nx; ++x) {
+                    const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
+                    tm[m * vol + i] = make_float2(h[m * vol + i], h[m * vol + i1]);
+                }
+        for (size_t zy = 0; zy < plane / d->nx * d->nz; ++zy)
+            for (int x = 0; x < d->nx; ++x) {
+                const size_t i = zy * d->nx + x, i1 = zy * d->nx + std::min(x + 1, d->nx - 1);
+                ed[i] = make_float4(E[i], E[i1], D[i], D[i1]);
+            }
+        CUDA_TRY(cudaMalloc(&ctx->d_tmap, sizeof(float2) * tm.size()));
+        CUDA_TRY(cudaMalloc(&ctx->d_ed, sizeof(float4) * ed.size()));
+        CUDA_TRY(cudaMemcpy(ctx->d_tmap, tm.data(), sizeof(float2) * tm.size(), cudaMemcpyHostToDevice));
+        CUDA_TRY(cudaMemcpy(ctx->d_ed, ed.data(), sizeof(float4) * ed.size(), cudaMemcpyHostToDevice));
+        g.tmap = (const float2*)ctx->d_tmap;
+        g.ed = (const float4*)ctx->d_ed;
+    }
+    g.layout = layout;
     g.nx = d->nx; g.ny = d->ny; g.nz = d->nz; g.n_type = nt;
     g.ox = d->origin[0]; g.oy = d->origin[1]; g.oz = d->origin[2];
     g.h = d->spacing;

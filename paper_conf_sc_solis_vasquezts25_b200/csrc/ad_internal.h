@@ -87,11 +87,19 @@ struct LigDev {
 // Grid in device memory, x-pair layout:
 //   tmap [n_type][nz][ny][nx] float2 (v[x], v[x+1])
 //   ed   [nz][ny][nx]         float4 (E[x], E[x+1], D[x], D[x+1])
+// Cell-record layout (layout == 1, used when it fits comfortably in L2): for every
+// cell (x,y,z) the 8 corner values, corner index dx + 2 dy + 4 dz:
+//   tc8 [n_type][nz][ny][nx][8]  (32 B, one 256-bit load per atom)
+//   ed8 [nz][ny][nx][16]         (E corners then D corners, 64 B, two 256-bit loads)
+// -> 3 loads / 96 B per atom = the algorithmic bytes, 8x the map memory.
 struct GridDev {
     const float2* tmap;
     const float4* ed;
+    const float* tc8;
+    const float* ed8;
     int32_t nx, ny, nz, n_type;
     float ox, oy, oz, h, inv_h;
+    int32_t layout;  // 0 = x-pair, 1 = cell records
 };
 
 // Per-warp scratch layout (offsets in bytes from the warp's slice; 16-aligned).

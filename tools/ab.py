@@ -39,9 +39,12 @@ def main():
         for v in variants:
             parts = v.split(":")
             lib, w, mode = parts[0], (parts[1] if len(parts) > 1 else "0") or "0", (parts[2] if len(parts) > 2 else "")
+            layout = parts[3] if len(parts) > 3 else ""
             env = dict(os.environ, AD_LIB=os.path.abspath(lib))
             if mode:
                 env["AD_INTRA_MODE"] = mode
+            if layout:
+                env["AD_GRID_LAYOUT"] = layout
             out = subprocess.check_output([sys.executable, "-c", CHILD, cfg, eng, w], env=env, text=True)
             d = json.loads(out.strip().splitlines()[-1])
             res[v] += d["ms"]
