@@ -193,8 +193,9 @@ typedef struct {
  *   best_energy  device [n_poses] FP32 best energy.
  *   run_best     device [n_poses/pop_per_run][1 + geno_stride] FP32 or NULL:
  *                per run the lowest best_energy (ties -> lowest pose index)
- *                followed by that pose's genes (O-8).  Requires
- *                n_poses % pop_per_run == 0.
+ *                followed by that pose's genes (O-8); columns past
+ *                6 + n_tors are 0 (single ligand) or the pose row's padding
+ *                (pose_ligand != NULL).  Requires n_poses % pop_per_run == 0.
  *   n_evals      device int64 accumulator or NULL; += n_poses * max_iters.
  * Errors: AD_ERR_INVALID_ARG, AD_ERR_STATE, AD_ERR_CUDA. */
 int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses,

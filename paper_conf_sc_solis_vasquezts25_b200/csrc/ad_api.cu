@@ -52,7 +52,8 @@ int32_t fail(int32_t code, const char* fmt, ...) {
 struct LigSlot {
     unsigned char* d_blob = nullptr;
     int32_t blob_bytes = 0;
-    int32_t scratch_bytes = 0;   // per warp (SIMT/TC)
+    int32_t scratch_bytes = 0;   // per warp (TC engine)
+    int32_t scratch_simt = 0;    // per warp (SIMT engine)
     int32_t block_scratch = 0;   // per block (baseline)
     int32_t n_atoms = 0, n_tors = 0;
     bool live = false;
@@ -78,6 +79,8 @@ struct ad_context {
     // faster on config 2: 1.40e8 vs 1.26e8 evals/s, profiles/README.md)
     int intra_mode = INTRA_SCATTER;
     int32_t last_grid = 0, last_block = 0, last_smem = 0;
+    // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
+    int32_t pairs_smem_max = 16384;
 };
 
 namespace {
@@ -115,7 +118,7 @@ int32_t sync_ligtab(ad_context* ctx) {
     std::vector<LigDev> h(n);
     for (int i = 0; i < n; ++i)
         h[i] = LigDev{ctx->ligs[i].live ? ctx->ligs[i].d_blob : nullptr, ctx->ligs[i].blob_bytes,
-                      ctx->ligs[i].scratch_bytes};
+                      ctx->ligs[i].scratch_bytes, ctx->ligs[i].scratch_simt, 0};
     if (n) CUDA_TRY(cudaMemcpy(ctx->d_ligtab, h.data(), sizeof(LigDev) * n, cudaMemcpyHostToDevice));
     return AD_OK;
 }
@@ -143,6 +146,9 @@ uint32_t swap_ij(uint32_t r) {
     const uint32_t i = r & 0xff, j = (r >> 8) & 0xff, si = (r >> 16) & 0xf, sj = (r >> 20) & 0xf;
     return j | (i << 8) | (sj << 16) | (si << 20) | (r & 0xff000000u);
 }
+
+// row stride (float4) of the gradient slots (a multiple of 8, ad_internal.h)
+int npad_of(int n_atoms) { return (n_atoms + 7) & ~7; }
 
 // Place the (<= 64) pairs of one step into 8 groups of 8 consecutive entries
 // (= the quarter-warps of the two sub-steps, the unit in which a 128-bit shared
@@ -223,6 +229,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         std::swap(perm[q], perm[(int)(st % (uint64_t)(q + 1))]);
     }
     const int kmax = std::min(8, std::max(2, 256 / std::max(n_atoms, 1)));
+    std::vector<std::vector<std::pair<int, uint32_t>>> best_rounds;
     for (int K = 1; K <= kmax; ++K) {
         std::vector<int> rem = perm;
         std::vector<std::vector<std::pair<int, uint32_t>>> rounds;
@@ -250,20 +257,21 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         if (R < best.rounds) {
             best.rounds = R;
             best.slots = K;
-            best.rec.assign((size_t)R * kPairsPerStep, 0u);  // i == j == 0 -> empty slot
-            best.dsv.assign((size_t)R * kPairsPerStep, 0.f);
-            // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
-            for (int r = 0; r < R; ++r) {
-                const std::vector<std::pair<int, uint32_t>> lay = arrange_step(rounds[r], n_atoms, K);
-                for (int l = 0; l < kPairsPerStep; ++l) {
-                    best.rec[(size_t)r * kPairsPerStep + l] = lay[l].second;
-                    best.dsv[(size_t)r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
-                }
-            }
+            best_rounds = std::move(rounds);
         }
         if (R <= target) break;
     }
     (void)target;
+    // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
+    best.rec.assign((size_t)best_rounds.size() * kPairsPerStep, 0u);
+    best.dsv.assign((size_t)best_rounds.size() * kPairsPerStep, 0.f);
+    for (size_t r = 0; r < best_rounds.size(); ++r) {
+        const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots);
+        for (int l = 0; l < kPairsPerStep; ++l) {
+            best.rec[r * kPairsPerStep + l] = lay[l].second;
+            best.dsv[r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
+        }
+    }
     if (P == 0) {
         best.rounds = 0;
         best.slots = 1;
@@ -471,6 +479,7 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
     ad_context* ctx = new (std::nothrow) ad_context();
     if (!ctx) return fail(AD_ERR_OOM, "host allocation failed");
     ctx->device = cuda_device;
+    if (const char* m = getenv("AD_PAIRS_SMEM_MAX")) ctx->pairs_smem_max = atoi(m);
     if (const char* m = getenv("AD_INTRA_MODE"))
         ctx->intra_mode = strcmp(m, "owner") == 0 ? INTRA_OWNER : strcmp(m, "hybrid") == 0 ? INTRA_HYBRID : INTRA_SCATTER;
     cudaError_t e = cudaSetDevice(cuda_device);
@@ -763,7 +772,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     LigHeader H{};
     H.n_atoms = N; H.n_tors = T; H.n_pairs = P; H.n_types = nt;
     H.n_rounds = sch.rounds; H.n_slots = sch.slots; H.n_chain = (int)chain.size();
-    H.n_pad = (N + 7) & ~7;
+    H.n_pad = npad_of(N);  // gradient-slot row stride
     H.intra_mode = mode;
     H.n_entries = own.E;
     H.n_chunks = own.C;
@@ -788,8 +797,6 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.off_tinfo = B.put(tinfo.data(), sizeof(int4) * T);
     H.off_chain = B.put(chain.data(), chain.size());
     H.off_mask = B.put(mask.data(), sizeof(uint2) * N);
-    H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
-    H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
     // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
     // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
     std::vector<float4> tp8(tp.size() * AD_TP_COPIES);
@@ -798,15 +805,31 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.off_tp = B.put(tp8.data(), sizeof(float4) * tp8.size());
     H.off_comb = B.put(own.comb.data(), sizeof(int2) * own.comb.size());
     H.off_combidx = B.put(own.combidx.data(), sizeof(uint16_t) * own.combidx.size());
+    // the pair schedule goes last: large schedules stay in global memory (read
+    // through L1, one copy per SM) instead of being staged into every CTA
+    H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
+    H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
     H.blob_bytes = (int32_t)B.buf.size();
+    const int32_t pair_bytes = H.blob_bytes - H.off_prec;
+    H.pairs_gmem = pair_bytes > ctx->pairs_smem_max ? 1 : 0;
+    if (const char* dump = getenv("AD_DUMP_SCHEDULE")) {  // debugging aid: raw schedule records
+        if (FILE* f = fopen(dump, "ab")) {
+            const int32_t hdr[4] = {N, sch.rounds, sch.slots, H.n_pad};
+            fwrite(hdr, sizeof(hdr), 1, f);
+            fwrite(sch.rec.data(), sizeof(uint32_t), sch.rec.size(), f);
+            fclose(f);
+        }
+    }
+    H.stage_bytes = H.pairs_gmem ? H.off_prec : H.blob_bytes;
     const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
     H.scratch_bytes = ws.bytes;
     memcpy(B.buf.data(), &H, sizeof(H));
 
     if (int32_t rc = set_device(ctx)) return rc;
     LigSlot s;
-    s.blob_bytes = H.blob_bytes;
+    s.blob_bytes = H.stage_bytes;  // shared-memory bytes staged per CTA
     s.scratch_bytes = ws.bytes;
+    s.scratch_simt = ws.bytes_simt;
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
@@ -854,12 +877,14 @@ int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const 
 
 // Choose warps per CTA: the most resident warps per SM, ties -> fewer warps per CTA
 // (finer load balance across SMs).
-int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int req_warps, cudaStream_t st) {
+int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int req_warps, cudaStream_t st,
+                    bool tc_engine) {
+    if (!tc_engine) L.scratch_bytes = L.scratch_simt;
     if (p.pose_ligand) {  // any live ligand may be referenced: size for the largest footprint
         for (const LigSlot& o : ctx->ligs)
             if (o.live) {
                 L.blob_bytes = std::max(L.blob_bytes, o.blob_bytes);
-                L.scratch_bytes = std::max(L.scratch_bytes, o.scratch_bytes);
+                L.scratch_bytes = std::max(L.scratch_bytes, tc_engine ? o.scratch_bytes : o.scratch_simt);
             }
     }
     // Every pose costs the same, so the launch is scored by (fewest waves of CTAs,
@@ -867,7 +892,7 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // launches keep power-of-two CTA sizes (pose_ligand groups must stay aligned).
     int best_w = 0, best_active = -1, best_waves = 1 << 30;
     size_t best_smem = 0;
-    for (int w = 1; w <= 8; ++w) {
+    for (int w = 1; w <= 16; ++w) {
         if (req_warps > 0 && w != req_warps) continue;
         if (p.pose_ligand && (w & (w - 1))) continue;
         const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
@@ -936,7 +961,7 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
     p.aux = aux;
     const bool want_grad = grad != nullptr || aux != nullptr;
     return launch_warp(ctx, ctx->ligs[lig], pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false), p, 0,
-                       (cudaStream_t)stream);
+                       (cudaStream_t)stream, false);
 }
 
 int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses, float* genes,
@@ -988,13 +1013,18 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         CUDA_TRY(cudaGetLastError());
     } else {
         int w = prm->warps_per_cta;
-        if (w < 0 || w > 8) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..8", w);
-        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st)) return rc;
+        if (w < 0 || w > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..16", w);
+        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st,
+                                     prm->engine == AD_ENGINE_TC))
+            return rc;
     }
     if (run_best) {
         const int runs = n_poses / prm->pop_per_run;
-        k_best_of_run<<<(runs + 3) / 4, 128, 0, st>>>(best_energy, genes, geno_stride, 6 + L.n_tors,
-                                                      prm->pop_per_run, runs, run_best);
+        // the whole genotype row is copied: with pose_ligand the runs of one call
+        // belong to ligands with different gene counts
+        k_best_of_run<<<(runs + 3) / 4, 128, 0, st>>>(best_energy, genes, geno_stride,
+                                                      pose_ligand ? geno_stride : 6 + L.n_tors, prm->pop_per_run,
+                                                      runs, run_best);
         CUDA_TRY(cudaGetLastError());
     }
     return AD_OK;
@@ -1031,6 +1061,29 @@ int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int3
         return fail(AD_ERR_INVALID_ARG, "unknown engine %d", engine);
     }
     CUDA_TRY(cudaGetLastError());
+    return AD_OK;
+}
+
+// Host-only inspection hook (not part of include/ad.h; no GPU needed): run the
+// intra-pair scheduler on a pair list of atoms 0..n_atoms-1.  Writes the number of
+// steps and slots; copies up to `cap` records (64 per step) to out_rec.
+int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pairs, int32_t* out_steps,
+                           int32_t* out_slots, uint32_t* out_rec, int32_t cap) {
+    if (n_atoms < 1 || n_atoms > AD_MAX_ATOMS || n_pairs < 0 || (n_pairs && !pairs) || !out_steps || !out_slots)
+        return fail(AD_ERR_INVALID_ARG, "bad arguments");
+    std::vector<int> pi(n_pairs), pj(n_pairs), ptp(n_pairs, 0);
+    std::vector<float> pd(n_pairs, 0.f);
+    for (int q = 0; q < n_pairs; ++q) {
+        pi[q] = pairs[2 * q];
+        pj[q] = pairs[2 * q + 1];
+        if (pi[q] < 0 || pi[q] >= n_atoms || pj[q] < 0 || pj[q] >= n_atoms || pi[q] == pj[q])
+            return fail(AD_ERR_INVALID_ARG, "bad pair %d", q);
+    }
+    const Schedule s = schedule_pairs(n_atoms, pi, pj, ptp, pd);
+    *out_steps = s.rounds;
+    *out_slots = s.slots;
+    if (out_rec)
+        for (int q = 0; q < std::min<int>(cap, (int)s.rec.size()); ++q) out_rec[q] = s.rec[q];
     return AD_OK;
 }
 

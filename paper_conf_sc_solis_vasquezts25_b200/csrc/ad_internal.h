@@ -4,7 +4,7 @@
 // shared memory with a single TMA bulk copy (cp.async.bulk) and keeps for all
 // max_iters ADADELTA iterations.  Layout (offsets in LigHeader, bytes):
 //
-//   LigHeader                                   144 B
+//   LigHeader                                   176 B
 //   atoms   float4 [N]      reference x,y,z (A, DFS order), charge q
 //   info    int2   [N]      {map | type<<8 | chain_len<<16, chain_start}
 //   tors    float4 [T][2]   reference-frame axis point P_b and unit axis u_b
@@ -73,15 +73,18 @@ struct alignas(16) LigHeader {
     int32_t off_chain, off_mask, off_prec, off_pdsv;    // 64
     int32_t off_tp, scratch_bytes, n_pad, intra_mode;   // 80
     int32_t n_entries, n_chunks, off_comb, off_combidx; // 96  (owner mode: E per lane, chunks per lane)
-    float ff[FF_N];                                     // 160
+    int32_t pairs_gmem, stage_bytes, reserved0, reserved1;  // 112: schedule in global memory?, bytes staged to smem
+    float ff[FF_N];                                     // 176
 };
-static_assert(sizeof(LigHeader) == 160, "header size");
+static_assert(sizeof(LigHeader) == 176, "header size");
 
 // Device table entry, one per uploaded ligand.
 struct LigDev {
-    const unsigned char* blob;
-    int32_t blob_bytes;
-    int32_t scratch_bytes;
+    const unsigned char* blob;  // global copy of the whole blob
+    int32_t blob_bytes;         // bytes staged into shared memory (header .. tables [.. schedule])
+    int32_t scratch_bytes;      // per-warp scratch, TC engine
+    int32_t scratch_simt;       // per-warp scratch, SIMT engine (no D tile)
+    int32_t pad;
 };
 
 // Grid in device memory, x-pair layout:
@@ -112,6 +115,7 @@ struct WarpScratch {
     int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
     int32_t genes;  // float  [64]
     int32_t part;   // float4 [C][32]       owner mode: per-(lane, chunk) partial gradients
+    int32_t bytes_simt;
     int32_t bytes;
 };
 
@@ -124,13 +128,16 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
     int32_t o = 0;
     s.x = o;     o += 16 * npad;
-    s.g = o;     o += 16 * npad * (n_slots + 1);  // + spare row targeted by empty schedule places
+    // rows of npad float4 (slot k of atom a at k * npad + a) + a spare row targeted
+    // by empty schedule places
+    s.g = o;     o += 16 * npad * (n_slots + 1);
     s.w = o;     o += 32 * (npad + 1);
-    s.d = o;     o += align16(4 * 8 * mpad);
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
     s.genes = o; o += 4 * kMaxGenes;
     s.part = o;  o += 16 * 32 * n_chunks;
+    s.bytes_simt = o;                               // the SIMT engine needs no D tile
+    s.d = o;     o += align16(4 * 8 * mpad);
     s.bytes = o;
     return s;
 }

@@ -40,6 +40,8 @@ def test_screen_matches_single_ligand_runs():
             out = ctx.local_search(lid, g, max_iters=iters, pop_per_run=pop)
             rb = out["run_best"].cpu().numpy()
             for r in range(runs):
-                assert np.array_equal(got[(k, r)], rb[r]), (k, r)
+                G1 = 1 + L.n_genes  # energy + this ligand's genes (padding columns differ by design)
+                bad = np.nonzero(got[(k, r)][:G1] != rb[r][:G1])[0]
+                assert bad.size == 0, (k, r, L.n_tors, bad, got[(k, r)][bad], rb[r][bad])
     finally:
         ctx.close()
