@@ -55,7 +55,14 @@ enum ad_engine {
      * tensor-core reduction of all seven values (ones-row MMA, Eq 1 generalised)
      * with the TF32 hi/lo error correction: the paper's TCEC in its
      * own design context (local search only). */
-    AD_ENGINE_PAPER_TCEC = 3
+    AD_ENGINE_PAPER_TCEC = 3,
+    /* NEXT-2 accuracy study: the warp-per-pose kernel with every sum (energy and
+     * D = M_ext * W) on the tensor cores in FP16 WITHOUT error correction: FP16
+     * operands and an FP16 accumulator kept inside the tensor core across
+     * k-steps (mma.sync m16n8k16 .f16.f16.f16.f16) -- the Schieffer-Peng
+     * reduction the paper starts from (Lst 1 bottom), whose
+     * accuracy loss (Fig 1) motivates TCEC.  Not for production use. */
+    AD_ENGINE_TC_FP16 = 4
 };
 
 /* Compile-time limits (violations return AD_ERR_LIMIT). */
@@ -179,7 +186,7 @@ typedef struct {
     float rho, eps;         /* decay and conditioning constants (0.8, 0.01; Z14) */
     int32_t pop_per_run;    /* poses per run for run_best; 0 = no run_best */
     int32_t engine;         /* enum ad_engine */
-    int32_t warps_per_cta;  /* poses per CTA for SIMT/TC (0 = library choice);
+    int32_t warps_per_cta;  /* poses per CTA for SIMT/TC/TC_FP16, 0..16 (0 = library choice);
                                threads per block for PAPER_BASELINE (0 = 64) */
     float* trace;           /* optional device [n_poses][max_iters][1 + 2*geno_stride]:
                                per evaluation E, genes, gradient (Z19 shadowed parity) */
@@ -209,7 +216,9 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
  *   engine    AD_ENGINE_SIMT (warp transpose-butterfly + one smem exchange),
  *             AD_ENGINE_TC (ones-vector TF32 MMA, hi/lo split, RN accumulation
  *             outside the tensor core), AD_ENGINE_PAPER_BASELINE (n_comp
- *             sequential block reductions with barriers).
+ *             sequential block reductions with barriers), AD_ENGINE_TC_FP16
+ *             (ones-vector FP16 MMA with the FP16 accumulator inside the tensor
+ *             core, per-warp results combined in FP16: no EC, NEXT-2).
  * n_partials in {32, 64, ..., 1024} (multiple of 32), n_comp in 1..64. */
 int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
                          const float* partials, float* out, void* cuda_stream);

@@ -17,9 +17,9 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("AD_LIB", os.path.join(PKG, "libad.so"))  # AD_LIB: A/B builds
 
 AD_OK, AD_ERR_INVALID_ARG, AD_ERR_LIMIT, AD_ERR_CUDA, AD_ERR_OOM, AD_ERR_STATE = 0, -1, -2, -3, -4, -5
-AD_ENGINE_SIMT, AD_ENGINE_TC, AD_ENGINE_PAPER_BASELINE, AD_ENGINE_PAPER_TCEC = 0, 1, 2, 3
+AD_ENGINE_SIMT, AD_ENGINE_TC, AD_ENGINE_PAPER_BASELINE, AD_ENGINE_PAPER_TCEC, AD_ENGINE_TC_FP16 = 0, 1, 2, 3, 4
 ENGINES = {"simt": AD_ENGINE_SIMT, "tc": AD_ENGINE_TC, "paper": AD_ENGINE_PAPER_BASELINE,
-           "paper_tcec": AD_ENGINE_PAPER_TCEC}
+           "paper_tcec": AD_ENGINE_PAPER_TCEC, "tc_fp16": AD_ENGINE_TC_FP16}
 
 # names exported by include/ad.h (tests check the .so exports all of them)
 EXPORTS = ("ad_last_error", "ad_version", "ad_context_create", "ad_context_destroy", "ad_upload_grids",

@@ -12,12 +12,15 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <array>
+#include <atomic>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
 #include <new>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "ad.h"
@@ -56,6 +59,7 @@ struct LigSlot {
     int32_t scratch_simt = 0;    // per warp (SIMT engine)
     int32_t block_scratch = 0;   // per block (baseline)
     int32_t n_atoms = 0, n_tors = 0;
+    float ff[FF_N] = {};         // LigHeader::ff (kernel parameters of every launch)
     bool live = false;
 };
 
@@ -150,6 +154,67 @@ uint32_t swap_ij(uint32_t r) {
 // row stride (float4) of the gradient slots (a multiple of 8, ad_internal.h)
 int npad_of(int n_atoms) { return (n_atoms + 7) & ~7; }
 
+// Shared-memory wavefronts of one group of 8 consecutive schedule entries (a
+// quarter-warp: the unit in which a 128-bit LDS/STS is serviced, confirmed by ncu
+// per-line wavefront counts on configs 2 and 3): for each of the four 128-bit
+// accesses of the pair loop (X_i, X_j and the two gradient targets slot * npad +
+// atom) the largest number of distinct 16-byte addresses sharing a bank group
+// (address / 16 mod 8).  1 per access = conflict free.
+int group_cost(const std::pair<int, uint32_t>* e, int npad) {
+    int cost = 0;
+    for (int acc = 0; acc < 4; ++acc) {
+        int addr[8], n = 0;
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t r = e[k].second;
+            const int i = r & 0xff, j = (r >> 8) & 0xff, si = (r >> 16) & 0xf, sj = (r >> 20) & 0xf;
+            const int a = acc == 0 ? i : acc == 1 ? j : acc == 2 ? si * npad + i : sj * npad + j;
+            bool seen = false;
+            for (int t = 0; t < n; ++t) seen |= addr[t] == a;
+            if (!seen) addr[n++] = a;
+        }
+        int per[8] = {0, 0, 0, 0, 0, 0, 0, 0}, mx = 1;
+        for (int t = 0; t < n; ++t) mx = std::max(mx, ++per[addr[t] & 7]);
+        cost += mx;
+    }
+    return cost;
+}
+
+// Local search over the placement of one step's 64 entries under group_cost:
+// swap two entries of different groups, or flip an entry's i/j orientation, when
+// that does not raise the cost (deterministic xorshift stream; the set of pairs
+// and their gradient slots is unchanged).
+void refine_step(std::vector<std::pair<int, uint32_t>>& out, int npad, int iters) {
+    uint64_t st = 0x2545F4914F6CDD1Dull;
+    auto rnd = [&]() { st ^= st << 13; st ^= st >> 7; st ^= st << 17; return st; };
+    int cost[8], cur = 0;
+    for (int g = 0; g < 8; ++g) cur += cost[g] = group_cost(&out[g * 8], npad);
+    for (int it = 0; it < iters && cur > 32; ++it) {  // 32 = conflict free
+        const int a = (int)(rnd() % 64), b = (int)(rnd() % 64);
+        const int ga = a / 8, gb = b / 8;
+        const bool flip = (rnd() & 3) == 0;
+        const auto sa = out[a], sb = out[b];
+        if (flip) {
+            if (out[a].first < 0) continue;
+            out[a].second = swap_ij(out[a].second);
+        } else {
+            if (ga == gb) continue;
+            std::swap(out[a], out[b]);
+        }
+        const int ca = group_cost(&out[ga * 8], npad);
+        const int cb = flip ? 0 : group_cost(&out[gb * 8], npad);
+        const int before = cost[ga] + (flip ? 0 : cost[gb]);
+        const int after = ca + (flip ? 0 : cb);
+        if (after <= before) {
+            cost[ga] = ca;
+            if (!flip) cost[gb] = cb;
+            cur += after - before;
+        } else {
+            out[a] = sa;
+            out[b] = sb;
+        }
+    }
+}
+
 // Place the (<= 64) pairs of one step into 8 groups of 8 consecutive entries
 // (= the quarter-warps of the two sub-steps, the unit in which a 128-bit shared
 // load/store is serviced).  Within a group the first atoms should have distinct
@@ -158,7 +223,7 @@ int npad_of(int n_atoms) { return (n_atoms + 7) & ~7; }
 // slot*npad + atom with npad % 8 == 0) is bank-conflict free.  Greedy, with the
 // i/j orientation as a free choice; leftovers fill empty places (then conflicts
 // are allowed).  Returns 64 entries, first == -1 marks an empty place.
-std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms,
+std::vector<std::pair<int, uint32_t>> arrange_greedy(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms,
                                                    int K) {
     std::vector<std::pair<int, uint32_t>> out(kPairsPerStep, {-1, 0u});
     std::vector<char> taken(pool.size(), 0);
@@ -209,12 +274,273 @@ std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<i
     return out;
 }
 
-// Greedy packing of pairs into steps of 64 (2 per lane) where each atom occurs
-// at most K times per step; occurrence k of atom a in a step targets gradient
-// slot k, so all 128 read-modify-writes of a step hit distinct addresses.
-// Pairs are visited in a fixed pseudo-random order (consecutive pairs of the
-// input list share atoms and would saturate K early); K in 1..4 (shared memory
-// grows with K), the fewest rounds win, ties -> smaller K.
+// Bank-conflict-minimal placement of one step.  Residue = storage row mod 8 =
+// the bank group of every 128-bit access of an atom (X rows and gradient rows
+// slot * npad + row, npad % 8 == 0).  A group of 8 entries is conflict free iff
+// its 8 i-residues are distinct and its 8 j-residues are distinct, i.e. the group
+// is a perfect matching of the bipartite residue multigraph (i-res -> j-res).
+//   (1) orient every pair (the pair term is symmetric) so that each residue is an
+//       i-end and a j-end about equally often: Euler orientation (odd-degree
+//       residues joined to a virtual vertex, edges oriented along closed trails
+//       -> |out - in| <= 1 per residue);
+//   (2) residues that are still an i-end (j-end) more than 8 times set edges
+//       aside (they must share a group with an equal residue: one conflict each);
+//   (3) fill every residue up to out = in = 8 with empty places, which may join
+//       any two residues (they target the spare row K on both sides and are
+//       masked by that slot);
+//   (4) peel the 8-regular bipartite multigraph into 8 perfect matchings (Kuhn's
+//       augmenting paths; a regular bipartite multigraph always has one, Hall)
+//       = the 8 groups;
+//   (5) every set-aside edge replaces an empty place, preferring one whose
+//       j-residue (i-residue) it matches, so it adds one conflict, not two.
+// With at most 16 pair ends per residue in the step (schedule_pairs' cap) and a
+// balanced orientation nothing is set aside and the step is conflict free.
+bool arrange_matching(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms, int K,
+                      std::vector<std::pair<int, uint32_t>>& out) {
+    if (n_atoms < 8 || pool.size() > (size_t)kPairsPerStep) return false;
+    const int E = (int)pool.size();
+    // (1) orientation: edges between residues, vertex 8 = virtual
+    std::vector<int> au(E), av(E);
+    int deg[9] = {0};
+    for (int e = 0; e < E; ++e) {
+        au[e] = pool[e].second & 7u;
+        av[e] = (pool[e].second >> 8) & 7u;
+        deg[au[e]]++;
+        deg[av[e]]++;
+    }
+    for (int r = 0; r < 8; ++r)
+        if (deg[r] & 1) { au.push_back(r); av.push_back(8); }
+    const int EA = (int)au.size();
+    std::vector<std::vector<int>> inc(9);
+    for (int e = 0; e < EA; ++e) { inc[au[e]].push_back(e); inc[av[e]].push_back(e); }
+    std::vector<char> used(EA, 0), fwd(EA, 1);  // fwd: traversed au -> av
+    std::vector<size_t> ptr(9, 0);
+    for (int start = 0; start < 9; ++start) {
+        for (;;) {  // closed trails from `start` while it has unused edges
+            while (ptr[start] < inc[start].size() && used[inc[start][ptr[start]]]) ptr[start]++;
+            if (ptr[start] == inc[start].size()) break;
+            int v = start;
+            do {
+                while (used[inc[v][ptr[v]]]) ptr[v]++;  // every vertex has even unused degree
+                const int e = inc[v][ptr[v]];
+                used[e] = 1;
+                fwd[e] = au[e] == v;
+                v = fwd[e] ? av[e] : au[e];
+            } while (v != start);
+        }
+    }
+    int outd[8] = {0}, ind[8] = {0};
+    std::vector<uint32_t> rec;
+    std::vector<int> ids;
+    std::vector<std::pair<int, uint32_t>> aside;
+    for (int e = 0; e < E; ++e) {
+        const uint32_t r = fwd[e] ? pool[e].second : swap_ij(pool[e].second);
+        const int ro = r & 7u, ri = (r >> 8) & 7u;
+        // (2) over-full residues set the edge aside
+        if (outd[ro] == 8 || ind[ri] == 8) {
+            aside.push_back({pool[e].first, r});
+            continue;
+        }
+        outd[ro]++;
+        ind[ri]++;
+        rec.push_back(r);
+        ids.push_back(pool[e].first);
+    }
+    // (3) empty places: i-residue with an out deficit -> j-residue with an in deficit;
+    // rows 0..7 hold real atoms (balance_slots), their X rows are real positions
+    int ro = 0, ri = 0;
+    while ((int)rec.size() < kPairsPerStep) {
+        while (outd[ro] == 8) ++ro;
+        while (ind[ri] == 8) ++ri;
+        outd[ro]++;
+        ind[ri]++;
+        rec.push_back((uint32_t)ro | ((uint32_t)ri << 8) | ((uint32_t)K << 16) | ((uint32_t)K << 20));
+        ids.push_back(-1);
+    }
+    // (4) peel 8 perfect matchings
+    std::vector<int> bucket[8][8];
+    for (int e = 0; e < kPairsPerStep; ++e) bucket[rec[e] & 7u][(rec[e] >> 8) & 7u].push_back(e);
+    out.assign(kPairsPerStep, {-1, 0u});
+    struct Aug {
+        std::vector<int> (*b)[8];
+        int* mr;
+        bool* sn;
+        bool run(int x) {
+            for (int v = 0; v < 8; ++v) {
+                if (b[x][v].empty() || sn[v]) continue;
+                sn[v] = true;
+                if (mr[v] < 0 || run(mr[v])) { mr[v] = x; return true; }
+            }
+            return false;
+        }
+    };
+    for (int g = 0; g < 8; ++g) {
+        int match_r[8];  // right vertex -> left vertex
+        for (int v = 0; v < 8; ++v) match_r[v] = -1;
+        for (int u = 0; u < 8; ++u) {
+            bool seen[8] = {false, false, false, false, false, false, false, false};
+            Aug aug{bucket, match_r, seen};
+            if (!aug.run(u)) return false;  // cannot happen for a regular multigraph
+        }
+        for (int v = 0; v < 8; ++v) {
+            const int u = match_r[v];
+            const int e = bucket[u][v].back();
+            bucket[u][v].pop_back();
+            out[g * 8 + u] = {ids[e], rec[e]};
+        }
+    }
+    // (5) set-aside edges replace empty places (one conflict when a residue matches)
+    for (const auto& x : aside) {
+        const int xo = x.second & 7u, xi = (x.second >> 8) & 7u;
+        int best = -1, bscore = -1;
+        for (int q = 0; q < kPairsPerStep; ++q) {
+            if (out[q].first >= 0) continue;
+            const int sc = ((int)(out[q].second & 7u) == xo) + ((int)((out[q].second >> 8) & 7u) == xi);
+            if (sc > bscore) { bscore = sc; best = q; }
+        }
+        if (best < 0) return false;  // cannot happen: E <= 64
+        out[best] = x;
+    }
+    return true;
+}
+
+std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms,
+                                                   int K) {
+    // two candidates, the lower modelled cost wins: the matching construction (exact
+    // when the step's residues allow it) and the greedy grouping; both polished by
+    // the local search unless already conflict free
+    static const int refine_iters = getenv("AD_REFINE_ITERS") ? atoi(getenv("AD_REFINE_ITERS")) : 20000;
+    const int npad = npad_of(n_atoms);
+    auto total = [&](const std::vector<std::pair<int, uint32_t>>& o) {
+        int c = 0;
+        for (int g = 0; g < 8; ++g) c += group_cost(&o[g * 8], npad);
+        return c;
+    };
+    std::vector<std::pair<int, uint32_t>> m;
+    int cm = 1 << 30;
+    if (!getenv("AD_NO_MATCHING") && arrange_matching(pool, n_atoms, K, m)) {
+        cm = total(m);
+        if (cm > 32) {
+            refine_step(m, npad, refine_iters);
+            cm = total(m);
+        }
+        if (cm == 32 || getenv("AD_MATCHING_ONLY")) return m;  // 4 accesses x 8 groups x 1 wavefront
+    }
+    std::vector<std::pair<int, uint32_t>> g = arrange_greedy(pool, n_atoms, K);
+    refine_step(g, npad, refine_iters);
+    return total(g) < cm ? g : m;
+}
+
+// Storage row of every atom (INTRA_SCATTER): the row picks the bank group
+// (row mod 8) of the atom's X row and gradient rows.  A step can only be placed
+// conflict free (arrange_matching) when no bank group carries more than 16 pair
+// ends in it, so the bank groups should carry equal numbers of pair ends.  The
+// per-atom phases (pose, gradient sums) access atoms a = lane + 32 m, i.e. every
+// aligned octet of atoms within one quarter-warp: rows are therefore only
+// permuted WITHIN each octet (rows 8m .. 8m+7 stay the octet's, so those
+// accesses stay conflict free), heaviest atom of the octet to the least loaded
+// bank group so far.
+std::vector<int> balance_slots(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj) {
+    std::vector<int> slot(n_atoms);
+    for (int a = 0; a < n_atoms; ++a) slot[a] = a;
+    if (n_atoms < 8 || getenv("AD_NO_BALANCE")) return slot;
+    std::vector<int> ends(n_atoms, 0);
+    for (size_t q = 0; q < pi.size(); ++q) {
+        ends[pi[q]]++;
+        ends[pj[q]]++;
+    }
+    long load[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int base = 0; base < n_atoms; base += 8) {
+        const int n = std::min(8, n_atoms - base);
+        int ord[8];
+        for (int k = 0; k < n; ++k) ord[k] = base + k;
+        std::stable_sort(ord, ord + n, [&](int x, int y) { return ends[x] > ends[y]; });
+        bool taken[8] = {false, false, false, false, false, false, false, false};
+        for (int k = 0; k < n; ++k) {
+            int best = -1;
+            for (int r = 0; r < 8; ++r)
+                if (!taken[r] && (best < 0 || load[r] < load[best])) best = r;
+            taken[best] = true;
+            slot[ord[k]] = base + best;
+            load[best] += ends[ord[k]];
+        }
+    }
+    return slot;
+}
+
+// Swap pairs between steps (or move them into free places) until no bank group
+// (row mod 8) carries more than 16 pair ends in any step, keeping every atom at
+// most K times per step: arrange_matching can then place every step conflict
+// free.  Deterministic (fixed xorshift stream); returns the remaining overload.
+int rebalance_steps(std::vector<std::vector<int>>& steps, const std::vector<int>& pi, const std::vector<int>& pj,
+                    int n_idx, int K, long iters) {
+    const int R = (int)steps.size();
+    if (R < 2) return 0;
+    const int cap = 2 * kPairsPerStep / 8;
+    std::vector<std::vector<uint8_t>> cnt(R, std::vector<uint8_t>(n_idx, 0));
+    std::vector<std::array<int, 8>> deg(R);
+    auto over = [&](const std::array<int, 8>& d) {
+        int o = 0;
+        for (int r = 0; r < 8; ++r) o += std::max(0, d[r] - cap);
+        return o;
+    };
+    int total = 0;
+    for (int a = 0; a < R; ++a) {
+        deg[a].fill(0);
+        for (int q : steps[a]) {
+            cnt[a][pi[q]]++;
+            cnt[a][pj[q]]++;
+            deg[a][pi[q] & 7]++;
+            deg[a][pj[q] & 7]++;
+        }
+        total += over(deg[a]);
+    }
+    uint64_t st = 0xD1B54A32D192ED03ull;
+    auto rnd = [&]() { st ^= st << 13; st ^= st >> 7; st ^= st << 17; return st; };
+    for (long it = 0; it < iters && total > 0; ++it) {
+        const int A = (int)(rnd() % R), B = (int)(rnd() % R);
+        if (A == B || steps[A].empty()) continue;
+        if (over(deg[A]) == 0 && over(deg[B]) == 0) continue;
+        const int ia = (int)(rnd() % steps[A].size());
+        const int p = steps[A][ia];
+        // q = a pair of B, or (-1) a free place of B
+        const int nb = (int)steps[B].size() + (steps[B].size() < (size_t)kPairsPerStep ? 1 : 0);
+        const int ib = (int)(rnd() % nb);
+        const int q = ib < (int)steps[B].size() ? steps[B][ib] : -1;
+        // K limits after the exchange
+        auto ok_into = [&](int S, int in, int outp) {
+            const int a = pi[in], b = pj[in];
+            int ca = cnt[S][a] + 1, cb = cnt[S][b] + 1;
+            if (outp >= 0) {
+                if (pi[outp] == a || pj[outp] == a) ca--;
+                if (pi[outp] == b || pj[outp] == b) cb--;
+            }
+            return ca <= K && cb <= K;
+        };
+        if (!ok_into(B, p, q) || (q >= 0 && !ok_into(A, q, p))) continue;
+        std::array<int, 8> dA = deg[A], dB = deg[B];
+        dA[pi[p] & 7]--; dA[pj[p] & 7]--; dB[pi[p] & 7]++; dB[pj[p] & 7]++;
+        if (q >= 0) { dB[pi[q] & 7]--; dB[pj[q] & 7]--; dA[pi[q] & 7]++; dA[pj[q] & 7]++; }
+        const int before = over(deg[A]) + over(deg[B]), after = over(dA) + over(dB);
+        if (after > before) continue;
+        // apply
+        cnt[A][pi[p]]--; cnt[A][pj[p]]--; cnt[B][pi[p]]++; cnt[B][pj[p]]++;
+        if (q >= 0) {
+            cnt[B][pi[q]]--; cnt[B][pj[q]]--; cnt[A][pi[q]]++; cnt[A][pj[q]]++;
+            steps[A][ia] = q;
+            steps[B][ib] = p;
+        } else {
+            steps[A][ia] = steps[A].back();
+            steps[A].pop_back();
+            steps[B].push_back(p);
+        }
+        deg[A] = dA;
+        deg[B] = dB;
+        total += after - before;
+    }
+    return total;
+}
+
 Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
                         const std::vector<int>& ptp, const std::vector<float>& pdsv) {
     const int P = (int)pi.size();
@@ -229,18 +555,29 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         std::swap(perm[q], perm[(int)(st % (uint64_t)(q + 1))]);
     }
     const int kmax = std::min(8, std::max(2, 256 / std::max(n_atoms, 1)));
+    const int n_idx = npad_of(n_atoms);  // atom indices are storage slots (< npad)
     std::vector<std::vector<std::pair<int, uint32_t>>> best_rounds;
+    // capped: at most 16 pair ends per bank group and step (arrange_matching's
+    // precondition); uncapped as a fallback when the cap costs a step
+    for (int capped = 1; capped >= 0; --capped)
     for (int K = 1; K <= kmax; ++K) {
+        if (!capped && best.rounds <= target) break;
         std::vector<int> rem = perm;
         std::vector<std::vector<std::pair<int, uint32_t>>> rounds;
-        std::vector<int> cnt(n_atoms);
+        std::vector<int> cnt(n_idx);
+        const int rcap = (capped && n_atoms >= 8) ? 2 * kPairsPerStep / 8 : 1 << 30;
         while (!rem.empty()) {
             std::fill(cnt.begin(), cnt.end(), 0);
+            int rc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             std::vector<std::pair<int, uint32_t>> rnd;
             std::vector<int> rest;
             for (int q : rem) {
                 const int i = pi[q], j = pj[q];
-                if ((int)rnd.size() < kPairsPerStep && cnt[i] < K && cnt[j] < K) {
+                const int need_i = 1 + ((i & 7) == (j & 7)), need_j = need_i;
+                if ((int)rnd.size() < kPairsPerStep && cnt[i] < K && cnt[j] < K && rc[i & 7] + need_i <= rcap &&
+                    rc[j & 7] + need_j <= rcap) {
+                    rc[i & 7]++;
+                    rc[j & 7]++;
                     const uint32_t r = (uint32_t)i | ((uint32_t)j << 8) | ((uint32_t)cnt[i] << 16) |
                                        ((uint32_t)cnt[j] << 20) | ((uint32_t)ptp[q] << 24);
                     cnt[i]++;
@@ -254,6 +591,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
             rem.swap(rest);
         }
         const int R = (int)rounds.size();
+        if (getenv("AD_DEBUG_SCHEDULE")) fprintf(stderr, "[libad] schedule capped=%d K=%d rounds=%d (target %d)\n", capped, K, R, target);
         if (R < best.rounds) {
             best.rounds = R;
             best.slots = K;
@@ -262,16 +600,46 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         if (R <= target) break;
     }
     (void)target;
+    if (n_atoms >= 8 && !getenv("AD_NO_REBALANCE")) {
+        // cross-step rebalancing, then slots re-assigned by occurrence order
+        std::vector<std::vector<int>> ids(best_rounds.size());
+        for (size_t r = 0; r < best_rounds.size(); ++r)
+            for (const auto& e : best_rounds[r]) ids[r].push_back(e.first);
+        const int left = rebalance_steps(ids, pi, pj, n_idx, best.slots, 200000L * (long)ids.size());
+        if (getenv("AD_DEBUG_SCHEDULE")) fprintf(stderr, "[libad] rebalance: overload left %d\n", left);
+        std::vector<int> cnt(n_idx);
+        for (size_t r = 0; r < ids.size(); ++r) {
+            std::fill(cnt.begin(), cnt.end(), 0);
+            best_rounds[r].clear();
+            for (int q : ids[r]) {
+                const int i = pi[q], j = pj[q];
+                best_rounds[r].push_back({q, (uint32_t)i | ((uint32_t)j << 8) | ((uint32_t)cnt[i] << 16) |
+                                                 ((uint32_t)cnt[j] << 20) | ((uint32_t)ptp[q] << 24)});
+                cnt[i]++;
+                cnt[j]++;
+            }
+        }
+    }
     // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
     best.rec.assign((size_t)best_rounds.size() * kPairsPerStep, 0u);
     best.dsv.assign((size_t)best_rounds.size() * kPairsPerStep, 0.f);
-    for (size_t r = 0; r < best_rounds.size(); ++r) {
-        const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots);
-        for (int l = 0; l < kPairsPerStep; ++l) {
-            best.rec[r * kPairsPerStep + l] = lay[l].second;
-            best.dsv[r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
+    // steps are arranged independently (deterministic per step): spread them over
+    // the host's cores
+    std::atomic<size_t> next{0};
+    auto worker = [&]() {
+        for (size_t r; (r = next.fetch_add(1)) < best_rounds.size();) {
+            const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots);
+            for (int l = 0; l < kPairsPerStep; ++l) {
+                best.rec[r * kPairsPerStep + l] = lay[l].second;
+                best.dsv[r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
+            }
         }
-    }
+    };
+    const size_t n_thr = std::min<size_t>(best_rounds.size(), std::max(1u, std::thread::hardware_concurrency()));
+    std::vector<std::thread> pool;
+    for (size_t t = 1; t < n_thr; ++t) pool.emplace_back(worker);
+    worker();
+    for (auto& t : pool) t.join();
     if (P == 0) {
         best.rounds = 0;
         best.slots = 1;
@@ -715,6 +1083,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     }
     if (nt * nt > 256) return fail(AD_ERR_LIMIT, "n_types^2 > 256");
     const int mode = ctx->intra_mode;
+    std::vector<int> slot(N);  // storage slot (X / gradient row) of every atom; identity unless balanced
+    for (int k = 0; k < N; ++k) slot[k] = k;
     Schedule sch;
     OwnerList own;
     if (mode == INTRA_OWNER) {
@@ -735,7 +1105,13 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         own.comb = std::move(hy.comb);
         own.combidx = std::move(hy.combidx);
     } else {
-        sch = schedule_pairs(N, pi, pj, ptp, pd);
+        slot = balance_slots(N, pi, pj);
+        std::vector<int> si(P), sj(P);
+        for (int q = 0; q < P; ++q) {
+            si[q] = slot[pi[q]];
+            sj[q] = slot[pj[q]];
+        }
+        sch = schedule_pairs(N, si, sj, ptp, pd);
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -752,7 +1128,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         for (int b = 0; b < T; ++b)
             if (M[b][a]) { ch.push_back(b); m |= 1ull << b; }
         std::sort(ch.begin(), ch.end(), [&](int x, int y) { return msize[x] < msize[y]; });  // leaf -> root
-        info[k] = make_int2(d->atom_map[a] | (d->atom_type[a] << 8) | ((int)ch.size() << 16), (int)chain.size());
+        info[k] = make_int2(d->atom_map[a] | (d->atom_type[a] << 8) | ((int)ch.size() << 16) | (slot[k] << 24),
+                            (int)chain.size());
         for (int b : ch) chain.push_back((uint8_t)b);
         mask[k] = make_uint2((uint32_t)m, (uint32_t)(m >> 32));
     }
@@ -766,7 +1143,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         if (!(nu > 0)) return fail(AD_ERR_INVALID_ARG, "torsion %d has a zero-length axis", b);
         tors[2 * b] = make_float4((float)P0[0], (float)P0[1], (float)P0[2], 0.f);
         tors[2 * b + 1] = make_float4((float)(u[0] / nu), (float)(u[1] / nu), (float)(u[2] / nu), 0.f);
-        tinfo[b] = make_int4(newi[a0], newi[c0], lo[b], hi[b]);
+        tinfo[b] = make_int4(slot[newi[a0]], slot[newi[c0]], lo[b], hi[b]);
     }
 
     LigHeader H{};
@@ -833,6 +1210,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
+    memcpy(s.ff, H.ff, sizeof(s.ff));
     CUDA_TRY(cudaMalloc(&s.d_blob, B.buf.size()));
     CUDA_TRY(cudaMemcpy(s.d_blob, B.buf.data(), B.buf.size(), cudaMemcpyHostToDevice));
     s.live = true;
@@ -860,7 +1238,9 @@ namespace {
 typedef void (*WarpKernel)(const KParams);
 
 WarpKernel pick_warp_kernel(int engine, bool grad, bool ls) {
-    if (ls) return engine == AD_ENGINE_TC ? k_warp_engine<1, true, true> : k_warp_engine<0, true, true>;
+    if (ls) return engine == AD_ENGINE_TC        ? k_warp_engine<1, true, true>
+                   : engine == AD_ENGINE_TC_FP16 ? k_warp_engine<2, true, true>
+                                                 : k_warp_engine<0, true, true>;
     if (!grad) return k_warp_engine<0, false, false>;
     return engine == AD_ENGINE_TC ? k_warp_engine<1, true, false> : k_warp_engine<0, true, false>;
 }
@@ -872,6 +1252,15 @@ int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const 
     if (n_poses < 0) return fail(AD_ERR_INVALID_ARG, "n_poses < 0");
     if (n_poses > 0 && !genes) return fail(AD_ERR_INVALID_ARG, "genes is NULL");
     if (stride < 6 + ctx->ligs[lig].n_tors) return fail(AD_ERR_INVALID_ARG, "geno_stride %d < 6 + n_tors", stride);
+    return AD_OK;
+}
+
+// pose_ligand launches may touch any live ligand; the scoring constants are kernel
+// parameters, so they must be identical across the live ligands
+int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
+    for (const LigSlot& o : ctx->ligs)
+        if (o.live && memcmp(o.ff, ctx->ligs[lig].ff, sizeof(o.ff)) != 0)
+            return fail(AD_ERR_INVALID_ARG, "pose_ligand launches need every live ligand uploaded with the same ad_ff_params");
     return AD_OK;
 }
 
@@ -939,6 +1328,7 @@ KParams base_params(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligan
     p.err = ctx->d_err;
     p.n_ligs = (int32_t)ctx->ligs.size();
     p.max_iters = 1;
+    p.pc = pair_const_from_ff(ctx->ligs[lig].ff);
     return p;
 }
 
@@ -951,6 +1341,9 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
                        void* stream) {
     if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
     if (n_poses > 0 && !energy) return fail(AD_ERR_INVALID_ARG, "energy is NULL");
+    if (pose_ligand) {
+        if (int32_t rc = check_common_ff(ctx, lig)) return rc;
+    }
     if (int32_t rc = set_device(ctx)) return rc;
     if (int32_t rc = check_device_err(ctx)) return rc;
     if (n_poses == 0) return AD_OK;
@@ -970,9 +1363,12 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
     if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
     if (prm->max_iters < 1) return fail(AD_ERR_INVALID_ARG, "max_iters must be >= 1");
-    if (prm->engine < 0 || prm->engine > 3) return fail(AD_ERR_INVALID_ARG, "unknown engine %d", prm->engine);
+    if (prm->engine < 0 || prm->engine > 4) return fail(AD_ERR_INVALID_ARG, "unknown engine %d", prm->engine);
     if (!(prm->rho >= 0.f && prm->rho < 1.f) || !(prm->eps > 0.f)) return fail(AD_ERR_INVALID_ARG, "need 0 <= rho < 1, eps > 0");
     if (n_poses > 0 && !best_energy) return fail(AD_ERR_INVALID_ARG, "best_energy is NULL");
+    if (pose_ligand) {
+        if (int32_t rc = check_common_ff(ctx, lig)) return rc;
+    }
     if (run_best && (prm->pop_per_run <= 0 || n_poses % prm->pop_per_run))
         return fail(AD_ERR_INVALID_ARG, "run_best needs pop_per_run > 0 dividing n_poses");
     if (int32_t rc = set_device(ctx)) return rc;
@@ -1015,7 +1411,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         int w = prm->warps_per_cta;
         if (w < 0 || w > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..16", w);
         if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st,
-                                     prm->engine == AD_ENGINE_TC))
+                                     prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16))
             return rc;
     }
     if (run_best) {
@@ -1055,6 +1451,12 @@ int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int3
         if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "TC reduce staging too large");
         CUDA_TRY(cudaFuncSetAttribute(k_reduce_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         k_reduce_tc<<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp);
+    } else if (engine == AD_ENGINE_TC_FP16) {
+        const int c8 = (n_comp + 7) & ~7;
+        const size_t smem = sizeof(float) * (size_t)nw * 32 * c8 + sizeof(uint16_t) * (size_t)nw * c8;
+        if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "TC reduce staging too large");
+        CUDA_TRY(cudaFuncSetAttribute(k_reduce_tc_fp16, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        k_reduce_tc_fp16<<<n_blocks, n_partials, smem, st>>>(partials, out, n_comp);
     } else if (engine == AD_ENGINE_PAPER_BASELINE) {
         k_reduce_paper<<<n_blocks, n_partials, 0, st>>>(partials, out, n_comp);
     } else {
@@ -1068,7 +1470,7 @@ int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int3
 // intra-pair scheduler on a pair list of atoms 0..n_atoms-1.  Writes the number of
 // steps and slots; copies up to `cap` records (64 per step) to out_rec.
 int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pairs, int32_t* out_steps,
-                           int32_t* out_slots, uint32_t* out_rec, int32_t cap) {
+                           int32_t* out_slots, uint32_t* out_rec, int32_t cap, int32_t* out_atom_slot) {
     if (n_atoms < 1 || n_atoms > AD_MAX_ATOMS || n_pairs < 0 || (n_pairs && !pairs) || !out_steps || !out_slots)
         return fail(AD_ERR_INVALID_ARG, "bad arguments");
     std::vector<int> pi(n_pairs), pj(n_pairs), ptp(n_pairs, 0);
@@ -1079,6 +1481,13 @@ int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
         if (pi[q] < 0 || pi[q] >= n_atoms || pj[q] < 0 || pj[q] >= n_atoms || pi[q] == pj[q])
             return fail(AD_ERR_INVALID_ARG, "bad pair %d", q);
     }
+    const std::vector<int> slot = balance_slots(n_atoms, pi, pj);
+    for (int q = 0; q < n_pairs; ++q) {
+        pi[q] = slot[pi[q]];
+        pj[q] = slot[pj[q]];
+    }
+    if (out_atom_slot)
+        for (int a = 0; a < n_atoms; ++a) out_atom_slot[a] = slot[a];
     const Schedule s = schedule_pairs(n_atoms, pi, pj, ptp, pd);
     *out_steps = s.rounds;
     *out_slots = s.slots;

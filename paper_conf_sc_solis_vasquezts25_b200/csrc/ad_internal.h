@@ -6,14 +6,15 @@
 //
 //   LigHeader                                   176 B
 //   atoms   float4 [N]      reference x,y,z (A, DFS order), charge q
-//   info    int2   [N]      {map | type<<8 | chain_len<<16, chain_start}
+//   info    int2   [N]      {map | type<<8 | chain_len<<16 | slot<<24, chain_start}; slot =
+//                           the atom's storage row in the per-pose X / gradient arrays
 //   tors    float4 [T][2]   reference-frame axis point P_b and unit axis u_b
-//   tinfo   int4   [T]      {a_b, c_b, lo_b, hi_b}: axis atoms and the moving set
+//   tinfo   int4   [T]      {a_b, c_b, lo_b, hi_b}: axis atoms (storage rows) and the moving set
 //                           M_b = [lo_b, hi_b) (contiguous thanks to DFS order)
 //   chain   u8     [Lrot]   per atom: the torsions moving it, leaf -> root
 //   mask    u32x2  [N]      per atom bitmask of torsions moving it (baseline engine)
 //   prec    u32    [R*64]   pair schedule: i | j<<8 | slot_i<<16 | slot_j<<20 | tp<<24
-//                           (i == j marks an empty slot).  Step r holds entries
+//                           (slot_i == K marks an empty place).  Step r holds entries
 //                           [64r, 64r+64): lane l takes 64r+l and 64r+32+l; within a
 //                           step every (slot, atom) target is distinct -> no atomics.
 //   pdsv    f32    [R*64]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
@@ -153,8 +154,9 @@ __host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, in
     BlockScratch s;
     int32_t o = 0;
     const int32_t t1 = n_tors > 0 ? n_tors : 1;
-    s.x = o;     o += 16 * n_atoms;
-    s.g = o;     o += 16 * n_atoms;
+    const int32_t npad = (n_atoms + 7) & ~7;  // rows are storage slots (< npad)
+    s.x = o;     o += 16 * npad;
+    s.g = o;     o += 16 * npad;
     s.trig = o;  o += align16(8 * (n_tors + 3));
     s.tw = o;    o += 32 * t1;
     s.tacc = o;  o += align16(4 * t1);
@@ -165,8 +167,35 @@ __host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, in
     return s;
 }
 
+// Scoring constants of the pair term and the out-of-grid weight, derived from a
+// ligand's LigHeader::ff on the host and passed as kernel parameters: the kernels
+// use them as constant-bank operands, so they occupy no registers in the pair loop.
+// Every ligand of one launch must share them (ad_api.cu checks on the host).
+struct PairConst {
+    float delta, cut_vdw, cut_el, rmin, A, B, k, nlB2, kBlB, coeff_el, ds_exp2, inv_s2, w_out;
+};
+
+__host__ __device__ inline PairConst pair_const_from_ff(const float* ff) {
+    PairConst c;
+    c.delta = ff[FF_DELTA];
+    c.cut_vdw = ff[FF_CUT_VDW];
+    c.cut_el = ff[FF_CUT_EL];
+    c.rmin = ff[FF_EL_RMIN];
+    c.A = ff[FF_DIEL_A];
+    c.B = ff[FF_DIEL_B];
+    c.k = ff[FF_DIEL_K];
+    c.nlB2 = -ff[FF_DIEL_LB] * 1.4426950408889634f;  // exp(-lB r) = ex2(nlB2 r)
+    c.kBlB = ff[FF_DIEL_K] * ff[FF_DIEL_B] * ff[FF_DIEL_LB];
+    c.coeff_el = ff[FF_COEFF_EL];
+    c.ds_exp2 = ff[FF_DS_EXP2];
+    c.inv_s2 = ff[FF_INV_S2];
+    c.w_out = ff[FF_W_OUT];
+    return c;
+}
+
 struct KParams {
     GridDev grid;
+    PairConst pc;
     const LigDev* ligs;
     int32_t lig;
     const int32_t* pose_ligand;

@@ -293,3 +293,65 @@ def test_reduction_engines_accuracy(ctx, ad, engine):
                 ex = np.array([[math.fsum(x[b, :, c].astype(np.float64)) for c in range(Cc)] for b in range(64)])
                 bound = (math.ceil(math.log2(P)) + 2) * 2.0 ** -24 * np.abs(x.astype(np.float64)).sum(axis=1)
                 assert np.all(np.abs(o - ex) <= bound), (P, Cc, dist)
+
+
+def test_reduction_fp16_no_ec_accuracy(ctx, ad):
+    """NEXT-2, config 4: the Schieffer-Peng FP16 reduction without EC (Lst 1
+    bottom) is correct to FP16 accuracy -- |S - S_exact| <=
+    (4 + n_warps) 2^-11 sum|x| -- and measurably worse than TCEC (the Fig 1 vs
+    Fig 3 finding, P:L177 / P:L199); large partials overflow FP16."""
+    import math
+    errs = {"tc": [], "tc_fp16": []}
+    for P in (128, 256, 1024):
+        Cc = 16
+        x = synth.make_reduction_partials(P * 7 + Cc, 64, P, Cc, "uniform")
+        xd = torch.from_numpy(x).cuda()
+        ex = np.array([[math.fsum(x[b, :, c].astype(np.float64)) for c in range(Cc)] for b in range(64)])
+        for eng in errs:
+            o = torch.empty(64, Cc, device="cuda")
+            ad.ad_reduce_blocks(ctx.h, ad.ENGINES[eng], xd, o)
+            torch.cuda.synchronize()
+            err = np.abs(o.cpu().numpy().astype(np.float64) - ex)
+            errs[eng].append(err.ravel())
+            if eng == "tc_fp16":
+                bound = (4 + P // 32) * 2.0 ** -11 * np.abs(x.astype(np.float64)).sum(axis=1)
+                assert np.all(err <= bound), P
+    e16, etc = np.concatenate(errs["tc_fp16"]), np.concatenate(errs["tc"])
+    assert np.median(e16) > 100 * max(np.median(etc), 1e-12)
+    # magnitudes beyond FP16's range (65504) overflow without EC / TF32's exponent
+    x = synth.make_reduction_partials(99, 8, 256, 8, "logmag")
+    o = torch.empty(8, 8, device="cuda")
+    ad.ad_reduce_blocks(ctx.h, ad.ENGINES["tc_fp16"], torch.from_numpy(x).cuda(), o)
+    torch.cuda.synchronize()
+    assert not np.all(np.isfinite(o.cpu().numpy()))
+
+
+def test_local_search_fp16_engine(ctx, cfg2):
+    """NEXT-2: the warp kernel with every sum on FP16 tensor cores without EC.
+    On relaxed poses (sums within FP16 range) energies stay within FP16
+    accumulation error of the oracle, and its gradient error is an order of
+    magnitude above the error-corrected TF32 engine's (P:L177 vs P:L199)."""
+    w = cfg2
+    (lid,) = _setup(ctx, w, "cfg2")
+    L = w.ligands[0]
+    Gn = L.n_genes
+    n = 64
+    # relax start poses with the TC engine first (clashing starts overflow FP16)
+    _, _, relaxed, _, _ = _ls(ctx, lid, w.genes[:n], "tc", 300)
+    res = {}
+    for eng in ("tc", "tc_fp16"):
+        tr, _, _, nev, _ = _ls(ctx, lid, relaxed, eng, 1)
+        assert nev == n
+        res[eng] = tr[:, 0]
+    stride = w.genes.shape[1]
+    Eo, Go, aux, ag = O.score(L, w.grid, w.ff, relaxed)
+    sc = energy_scale(aux)
+    e16 = res["tc_fp16"][:, 0].astype(np.float64)
+    assert np.all(np.isfinite(e16))
+    assert np.all(np.abs(e16 - Eo) <= 1e-3 + 2.0 ** -20 * sc + 34 * 2.0 ** -11 * aux[:, O.AUX_ABS_E])
+    rel = {}
+    for eng in res:
+        g = res[eng][:, 1 + stride:1 + stride + Gn].astype(np.float64)
+        rel[eng] = np.linalg.norm(g - Go[:, :Gn], axis=1) / np.maximum(np.linalg.norm(Go[:, :Gn], axis=1), 1e-6)
+    assert np.median(rel["tc_fp16"]) > 10 * np.median(rel["tc"])
+    assert np.median(rel["tc_fp16"]) < 0.05

@@ -22,25 +22,27 @@ def _schedule(lib, n_atoms, pairs):
     steps, slots = C.c_int32(), C.c_int32()
     cap = 64 * (len(pairs) + 64)
     rec = np.zeros(cap, np.uint32)
+    slot = np.zeros(max(n_atoms, 1), np.int32)
     rc = lib.adx_debug_schedule(n_atoms, len(pairs), pairs.ctypes.data_as(C.c_void_p), C.byref(steps),
-                                C.byref(slots), rec.ctypes.data_as(C.c_void_p), cap)
+                                C.byref(slots), rec.ctypes.data_as(C.c_void_p), cap, slot.ctypes.data_as(C.c_void_p))
     assert rc == 0
-    return steps.value, slots.value, rec[:steps.value * 64]
+    return steps.value, slots.value, rec[:steps.value * 64], slot[:n_atoms]
 
 
 @pytest.mark.parametrize("n_atoms,n_tors,seed", [(12, 2, 1), (40, 8, 2), (110, 32, 3), (70, 20, 4), (200, 4, 5)])
 def test_schedule_covers_pairs_with_distinct_targets(lib, n_atoms, n_tors, seed):
     L = synth.make_ligand(seed, n_atoms, n_tors, 8, chainlike=n_atoms > 80)
-    R, K, rec = _schedule(lib, L.n_atoms, L.pairs)
+    R, K, rec, slot = _schedule(lib, L.n_atoms, L.pairs)
+    npad = (L.n_atoms + 7) & ~7
+    assert sorted(slot.tolist()) == sorted(set(slot.tolist())) and slot.max() < npad   # injective storage rows
     assert R * 64 >= L.n_pairs and 1 <= K <= 8
     i, j = rec & 0xff, (rec >> 8) & 0xff
     si, sj = (rec >> 16) & 0xf, (rec >> 20) & 0xf
-    real = i != j
+    real = si != K                                                        # empty places: spare slot K
     got = sorted(tuple(sorted(p)) for p in zip(i[real].tolist(), j[real].tolist()))
-    assert got == sorted(tuple(sorted(p)) for p in L.pairs.tolist())      # every pair exactly once
+    assert got == sorted(tuple(sorted(p)) for p in slot[L.pairs].tolist())  # every pair exactly once
     assert np.all(si[real] < K) and np.all(sj[real] < K)
     assert np.all(si[~real] == K) and np.all(sj[~real] == K)             # empty places -> spare row
-    npad = (L.n_atoms + 7) & ~7
     for r in range(R):
         s = slice(64 * r, 64 * r + 64)
         m = real[s]
@@ -51,7 +53,32 @@ def test_schedule_covers_pairs_with_distinct_targets(lib, n_atoms, n_tors, seed)
 
 
 def test_schedule_empty_and_tiny(lib):
-    R, K, rec = _schedule(lib, 5, np.zeros((0, 2), np.int32))
+    R, K, rec, _ = _schedule(lib, 5, np.zeros((0, 2), np.int32))
     assert R == 0
-    R, K, rec = _schedule(lib, 2, [[0, 1]])
-    assert R == 1 and ((rec & 0xff) != ((rec >> 8) & 0xff)).sum() == 1
+    R, K, rec, _ = _schedule(lib, 2, [[0, 1]])
+    assert R == 1 and (((rec >> 16) & 0xf) != K).sum() == 1
+
+
+def _quarter_wavefronts(rec, npad):
+    """128-bit shared accesses are serviced per quarter-warp (8 lanes): wavefronts of
+    one access = max over bank groups (addr mod 8) of the distinct rows hit."""
+    i, j = rec & 0xff, (rec >> 8) & 0xff
+    si, sj = (rec >> 16) & 0xf, (rec >> 20) & 0xf
+    total = 0
+    for addr in (i, j, si * npad + i, sj * npad + j):
+        for g in range(0, len(rec), 8):
+            rows = set(addr[g:g + 8].tolist())
+            total += max(np.bincount([r % 8 for r in rows], minlength=8))
+    return total
+
+
+@pytest.mark.parametrize("cfg,max_ratio", [(2, 1.1), (3, 1.0)])
+def test_schedule_is_bank_conflict_free(lib, cfg, max_ratio):
+    """Residue balancing + cross-step rebalancing + matching placement: the pair
+    loop's X and gradient accesses hit (near) the ideal 1 wavefront per quarter-warp."""
+    L = synth.make_config(cfg).ligands[0]
+    R, K, rec, slot = _schedule(lib, L.n_atoms, L.pairs)
+    assert R <= -(-L.n_pairs // 64) + 2
+    npad = (L.n_atoms + 7) & ~7
+    ideal = 4 * len(rec) // 8
+    assert _quarter_wavefronts(rec, npad) <= max_ratio * ideal

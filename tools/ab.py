@@ -1,6 +1,6 @@
 """A/B timing of library builds / launch shapes / intra modes, interleaved subprocess runs.
 
-usage: python tools/ab.py CFG ENGINE LIB[:W[:MODE]] ...   (3 rounds x 5 timed launches each)
+usage: python tools/ab.py CFG ENGINE LIB[:W[:MODE[:LAYOUT[:NAME=VALUE...]]]] ...   (3 rounds x 5 timed launches each)
 Prints the median ms per LS launch (config CFG, full workload) per variant.
 """
 import json
@@ -45,6 +45,9 @@ def main():
                 env["AD_INTRA_MODE"] = mode
             if layout:
                 env["AD_GRID_LAYOUT"] = layout
+            for kv in parts[4:]:  # extra NAME=VALUE environment settings
+                k, _, val = kv.partition("=")
+                env[k] = val
             out = subprocess.check_output([sys.executable, "-c", CHILD, cfg, eng, w], env=env, text=True)
             d = json.loads(out.strip().splitlines()[-1])
             res[v] += d["ms"]
