@@ -209,6 +209,48 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
                         float* genes, int32_t geno_stride, float* best_energy, float* run_best, int64_t* n_evals,
                         const ad_ls_params* params, void* cuda_stream);
 
+/* NEXT-3: the Lamarckian GA around the local search (Alg 1).
+ * n_runs independent runs (coarse level) of pop_size individuals.  Each
+ * generation of an unfinished run: GA(population) -- elitism, binary tournaments
+ * (the better of two random individuals wins with probability tour_rate),
+ * two-point crossover (probability cross_rate), per-gene uniform mutation
+ * (probability mut_rate; +-dmov grid units on translation genes, +-dang degrees
+ * on angle genes) -- then the energy of every new individual, then
+ * LS(population): each individual with probability ls_rate runs ADADELTA
+ * (`ls`) and is replaced by its best genotype (Lamarckian).  A run
+ * stops when its evaluation count (pop per generation + LS individuals x
+ * ls.max_iters) reaches max_evals or its generation count reaches max_gens
+ * (2 500 000 and 27 000).  The operator parameters are not in the
+ * paper (DESIGN.md §7b readings; AutoDock-GPU defaults).  Random numbers: a
+ * counter-based SplitMix64 chain per (seed, generation, run, individual, draw),
+ * so results do not depend on launch shapes.
+ *   genes      device [n_runs * pop_size][geno_stride]: in = initial population,
+ *              out = final population (caller-owned)
+ *   energies   device [n_runs * pop_size]: out, final energies
+ *   run_best   device [n_runs][1 + geno_stride] or NULL: best energy + genes per run
+ *   n_evals    device int64 [n_runs] or NULL: evaluations per run
+ *   n_gens     device int32 [n_runs] or NULL: generations per run
+ * Blocks the calling thread until every run finished (one 4-byte read per
+ * generation); scratch is allocated per call.  Engines: SIMT, TC, TC_FP16. */
+typedef struct {
+    int32_t pop_size;       /* individuals per run (150) */
+    int32_t max_gens;       /* N_gens^MAX (27000) */
+    int64_t max_evals;      /* N_score-evals^MAX per run (2 500 000) */
+    int32_t elitism;        /* best individuals copied unchanged (1) */
+    float cross_rate;       /* 0.8 */
+    float mut_rate;         /* 0.02 per gene */
+    float tour_rate;        /* 0.6 */
+    float ls_rate;          /* 0.8 */
+    float dmov;             /* mutation half-width, translation genes, grid units */
+    float dang;             /* mutation half-width, angle genes, degrees (90) */
+    uint64_t seed;
+    ad_ls_params ls;        /* the local search (pop_per_run and trace ignored) */
+} ad_lga_params;
+
+int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* genes, int32_t geno_stride,
+                   float* energies, float* run_best, int64_t* n_evals, int32_t* n_gens, const ad_lga_params* params,
+                   void* cuda_stream);
+
 /* Reduction-engine microbenchmark (config 4; Eq 1-5): sum each of
  * n_comp components over n_partials per block.
  *   partials  device [n_blocks][n_partials][n_comp] FP32

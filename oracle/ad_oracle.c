@@ -544,4 +544,99 @@ double ado_exact_sum(const float* x, int64_t n, int64_t stride) {
     return s;
 }
 
+/* ---- NEXT-3: one generation of the Lamarckian GA (Alg 1) ----
+ * The paper names the operators (selection, crossover, mutation) and the
+ * driver loop, not their parameters; the readings (AutoDock-GPU
+ * defaults [ext]) are: elitism, binary tournaments (the better of two random
+ * individuals wins with probability tour_rate), two-point crossover with
+ * probability cross_rate, per-gene uniform mutation with probability mut_rate
+ * (+-dmov grid units on translation genes, +-dang degrees on angle genes), LS on
+ * each new individual with probability ls_rate.
+ *
+ * Random numbers: a counter-based generator (each side implements it; nothing
+ * is shared): x = mix(mix(mix(seed ^ (gen << 32 | run)) ^ (ind << 32 | d)))
+ * with mix = the SplitMix64 step (add the golden gamma, then the finaliser);
+ * a uniform u = (x >> 40) * 2^-24 (exact in FP32); an index = (x >> 32) % m.
+ * Draw ids d per new individual: 0/1/2 tournament 1 (a, b, coin), 3/4/5
+ * tournament 2, 6 crossover coin, 7/8 cut points, 16+i mutation coin of gene i,
+ * 80+i its delta, 150 LS coin.
+ * The mutation arithmetic is done in FP32 exactly as written (t = 2u - 1 is
+ * exact, delta = t * max one rounding, gene + delta one rounding): the genotype
+ * is FP32, so this reproduces the GPU bit for bit (compiled without
+ * contraction); selection compares the FP32 energies it is given. */
+static uint64_t ado_mix(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t ado_rng_mix(uint64_t z) { return ado_mix(z); }
+
+uint64_t ado_rng(uint64_t seed, uint32_t gen, uint32_t run, uint32_t ind, uint32_t d) {
+    return ado_mix(ado_mix(ado_mix(seed ^ (((uint64_t)gen << 32) | run)) ^ (((uint64_t)ind << 32) | d)));
+}
+
+static float ado_u24(uint64_t x) { return (float)(x >> 40) * (1.0f / 16777216.0f); }
+
+typedef struct {
+    int32_t pop, n_genes, stride, elitism;
+    float cross_rate, mut_rate, tour_rate, ls_rate;
+    float dmov, dang; /* mutation half-widths: grid units, degrees */
+} ado_ga;
+
+/* index of the better of a, b: lower energy, ties -> lower index */
+static int ado_better(const float* E, int a, int b) { return (E[a] < E[b] || (E[a] == E[b] && a < b)) ? a : b; }
+
+static int ado_tournament(const ado_ga* P, const float* E, uint64_t seed, uint32_t gen, uint32_t run, uint32_t ind,
+                          uint32_t d0) {
+    const int a = (int)((ado_rng(seed, gen, run, ind, d0) >> 32) % (uint64_t)P->pop);
+    const int b = (int)((ado_rng(seed, gen, run, ind, d0 + 1) >> 32) % (uint64_t)P->pop);
+    const int best = ado_better(E, a, b), worst = best == a ? b : a;
+    return ado_u24(ado_rng(seed, gen, run, ind, d0 + 2)) < P->tour_rate ? best : worst;
+}
+
+/* genes_in/out [pop][stride] of ONE run, E_in [pop] its energies. */
+int ado_ga_generation(const ado_ga* P, const float* genes_in, const float* E_in, float* genes_out, uint64_t seed,
+                      uint32_t gen, uint32_t run) {
+    const int pop = P->pop, G = P->n_genes, S = P->stride;
+    if (pop < 2 || G < 1 || G > 64 || S < G || P->elitism < 0 || P->elitism > pop) return -1;
+    /* elitism: the `elitism` best individuals, in order of increasing energy */
+    char* used = (char*)calloc((size_t)pop, 1);
+    for (int k = 0; k < P->elitism; k++) {
+        int bi = -1;
+        for (int q = 0; q < pop; q++)
+            if (!used[q] && (bi < 0 || ado_better(E_in, q, bi) == q)) bi = q;
+        used[bi] = 1;
+        memcpy(genes_out + (size_t)k * S, genes_in + (size_t)bi * S, sizeof(float) * (size_t)S);
+    }
+    free(used);
+    for (int k = P->elitism; k < pop; k++) {
+        const int p1 = ado_tournament(P, E_in, seed, gen, run, (uint32_t)k, 0);
+        const int p2 = ado_tournament(P, E_in, seed, gen, run, (uint32_t)k, 3);
+        float* c = genes_out + (size_t)k * S;
+        memcpy(c, genes_in + (size_t)p1 * S, sizeof(float) * (size_t)S);
+        if (ado_u24(ado_rng(seed, gen, run, (uint32_t)k, 6)) < P->cross_rate) {
+            int c1 = (int)((ado_rng(seed, gen, run, (uint32_t)k, 7) >> 32) % (uint64_t)(G + 1));
+            int c2 = (int)((ado_rng(seed, gen, run, (uint32_t)k, 8) >> 32) % (uint64_t)(G + 1));
+            if (c1 > c2) { int t = c1; c1 = c2; c2 = t; }
+            for (int i = c1; i < c2; i++) c[i] = genes_in[(size_t)p2 * S + i];
+        }
+        for (int i = 0; i < G; i++) {
+            if (!(ado_u24(ado_rng(seed, gen, run, (uint32_t)k, 16 + (uint32_t)i)) < P->mut_rate)) continue;
+            const float u = ado_u24(ado_rng(seed, gen, run, (uint32_t)k, 80 + (uint32_t)i));
+            const float t = 2.0f * u - 1.0f;
+            const float delta = t * (i < 3 ? P->dmov : P->dang);
+            c[i] = c[i] + delta;
+        }
+    }
+    return 0;
+}
+
+/* LS coin of every individual of one run: sel[k] = u < ls_rate (draw id 150). */
+int ado_ls_select(const ado_ga* P, uint64_t seed, uint32_t gen, uint32_t run, uint8_t* sel) {
+    for (int k = 0; k < P->pop; k++) sel[k] = ado_u24(ado_rng(seed, gen, run, (uint32_t)k, 150)) < P->ls_rate;
+    return 0;
+}
+
 int ado_version(void) { return 1; }

@@ -26,7 +26,7 @@ _lib = None
 def build(force: bool = False) -> str:
     """Compile the oracle with gcc (-O2, no fast-math, OpenMP)."""
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
-        cmd = ["gcc", "-O2", "-std=c11", "-fopenmp", "-fPIC", "-shared", "-Wall", "-o", LIB, SRC, "-lm"]
+        cmd = ["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared", "-Wall", "-o", LIB, SRC, "-lm"]
         subprocess.check_call(cmd)
     return LIB
 
@@ -64,6 +64,12 @@ def lib():
             L.ado_best_of_run.argtypes = [C.c_int32, C.c_int32, P, P]
             L.ado_exact_sum.argtypes = [P, C.c_int64, C.c_int64]
             L.ado_exact_sum.restype = C.c_double
+            L.ado_rng.argtypes = [C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32]
+            L.ado_rng.restype = C.c_uint64
+            L.ado_rng_mix.argtypes = [C.c_uint64]
+            L.ado_rng_mix.restype = C.c_uint64
+            L.ado_ga_generation.argtypes = [P, P, P, P, C.c_uint64, C.c_uint32, C.c_uint32]
+            L.ado_ls_select.argtypes = [P, C.c_uint64, C.c_uint32, C.c_uint32, P]
             _lib = L
     return _lib
 
@@ -168,6 +174,38 @@ def best_of_run(best_E, pop):
 def exact_sum(x: np.ndarray) -> float:
     x = np.ascontiguousarray(x, dtype=np.float32).reshape(-1)
     return float(lib().ado_exact_sum(_ptr(x), x.size, 1))
+
+
+class GA_(C.Structure):
+    _fields_ = [("pop", C.c_int32), ("n_genes", C.c_int32), ("stride", C.c_int32), ("elitism", C.c_int32),
+                ("cross_rate", C.c_float), ("mut_rate", C.c_float), ("tour_rate", C.c_float), ("ls_rate", C.c_float),
+                ("dmov", C.c_float), ("dang", C.c_float)]
+
+
+def ga_params(pop, n_genes, stride, elitism=1, cross_rate=0.8, mut_rate=0.02, tour_rate=0.6, ls_rate=0.8,
+              dmov=16.0, dang=90.0):
+    """NEXT-3 GA parameters (DESIGN.md 7b readings; dmov in grid units)."""
+    return GA_(pop, n_genes, stride, elitism, cross_rate, mut_rate, tour_rate, ls_rate, dmov, dang)
+
+
+def rng(seed, gen, run, ind, d) -> int:
+    """The counter-based generator of the GA (oracle side)."""
+    return int(lib().ado_rng(seed, gen, run, ind, d))
+
+
+def ga_generation(prm, genes, energies, seed, gen, run):
+    """One GA generation of one run: genes [pop, stride] f32, energies [pop] f32 -> new genes."""
+    genes = np.ascontiguousarray(genes, dtype=np.float32)
+    energies = np.ascontiguousarray(energies, dtype=np.float32)
+    out = np.zeros_like(genes)
+    assert lib().ado_ga_generation(C.byref(prm), _ptr(genes), _ptr(energies), _ptr(out), seed, gen, run) == 0
+    return out
+
+
+def ls_select(prm, seed, gen, run):
+    sel = np.zeros(prm.pop, dtype=np.uint8)
+    lib().ado_ls_select(C.byref(prm), seed, gen, run, _ptr(sel))
+    return sel.astype(bool)
 
 
 def _dummy_ff():

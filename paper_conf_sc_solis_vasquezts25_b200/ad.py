@@ -23,7 +23,7 @@ ENGINES = {"simt": AD_ENGINE_SIMT, "tc": AD_ENGINE_TC, "paper": AD_ENGINE_PAPER_
 
 # names exported by include/ad.h (tests check the .so exports all of them)
 EXPORTS = ("ad_last_error", "ad_version", "ad_context_create", "ad_context_destroy", "ad_upload_grids",
-           "ad_upload_ligand", "ad_free_ligand", "ad_score_poses", "ad_local_search", "ad_reduce_blocks",
+           "ad_upload_ligand", "ad_free_ligand", "ad_score_poses", "ad_local_search", "ad_lga_run", "ad_reduce_blocks",
            "ad_query", "ad_last_launch")
 
 
@@ -55,6 +55,12 @@ class LSParams(C.Structure):
                 ("engine", C.c_int32), ("warps_per_cta", C.c_int32), ("trace", C.c_void_p)]
 
 
+class LGAParams(C.Structure):
+    _fields_ = [("pop_size", C.c_int32), ("max_gens", C.c_int32), ("max_evals", C.c_int64), ("elitism", C.c_int32),
+                ("cross_rate", C.c_float), ("mut_rate", C.c_float), ("tour_rate", C.c_float), ("ls_rate", C.c_float),
+                ("dmov", C.c_float), ("dang", C.c_float), ("seed", C.c_uint64), ("ls", LSParams)]
+
+
 _lock = threading.Lock()
 _lib = None
 
@@ -79,6 +85,7 @@ def lib():
             L.ad_score_poses.argtypes = [P, I32, P, I32, P, I32, P, P, P, P]
             L.ad_local_search.argtypes = [P, I32, P, I32, P, I32, P, P, P, C.POINTER(LSParams), P]
             L.ad_reduce_blocks.argtypes = [P, I32, I32, I32, I32, P, P, P]
+            L.ad_lga_run.argtypes = [P, I32, I32, P, I32, P, P, P, P, C.POINTER(LGAParams), P]
             L.ad_query.argtypes = [P, I32, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
             L.ad_last_launch.argtypes = [P, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
             for name in EXPORTS:
@@ -179,6 +186,20 @@ def ad_local_search(ctx, lig, pose_ligand, genes, best_energy, run_best=None, n_
                                  _dptr(n_evals, torch.int64), C.byref(prm), _stream(stream)))
 
 
+def ad_lga_run(ctx, lig, n_runs, genes, energies, run_best=None, n_evals=None, n_gens=None, *, pop_size=150,
+               max_gens=27000, max_evals=2_500_000, elitism=1, cross_rate=0.8, mut_rate=0.02, tour_rate=0.6,
+               ls_rate=0.8, dmov=16.0, dang=90.0, seed=0, ls_iters=300, rho=0.8, eps=0.01, engine=AD_ENGINE_SIMT,
+               warps_per_cta=0, stream=None) -> None:
+    import torch
+    n, stride = genes.shape
+    assert n == n_runs * pop_size
+    prm = LGAParams(pop_size, max_gens, max_evals, elitism, cross_rate, mut_rate, tour_rate, ls_rate, dmov, dang,
+                    seed, LSParams(ls_iters, rho, eps, 0, engine, warps_per_cta, None))
+    _check(lib().ad_lga_run(ctx, lig, n_runs, _dptr(genes, torch.float32), stride, _dptr(energies, torch.float32),
+                            _dptr(run_best, torch.float32), _dptr(n_evals, torch.int64), _dptr(n_gens, torch.int32),
+                            C.byref(prm), _stream(stream)))
+
+
 def ad_reduce_blocks(ctx, engine, partials, out, stream=None) -> None:
     import torch
     nb, P, Cc = partials.shape
@@ -195,7 +216,14 @@ def ad_query(ctx, lig=-1):
 def ad_last_launch(ctx):
     a, b, c = C.c_int32(), C.c_int32(), C.c_int32()
     _check(lib().ad_last_launch(ctx, C.byref(a), C.byref(b), C.byref(c)))
-    return {"grid": a.value, "block": b.value, "smem_bytes": c.value}
+    out = {"grid": a.value, "block": b.value, "smem_bytes": c.value}
+    try:  # inspection hook, not part of include/ad.h
+        f = lib().adx_last_maxreg
+        f.argtypes, f.restype = [C.c_void_p], C.c_int32
+        out["maxreg"] = int(f(ctx))
+    except AttributeError:
+        pass
+    return out
 
 
 # ---------------------------------------------------------------- convenience
@@ -250,3 +278,16 @@ class Context:
                         pop_per_run=pop_per_run, engine=ENGINES[engine] if isinstance(engine, str) else engine,
                         warps_per_cta=warps_per_cta, trace=tr)
         return {"best_energy": bE, "run_best": rb, "trace": tr}
+
+    def lga(self, lig_id, genes, n_runs, *, engine="simt", **kw):
+        """NEXT-3 Lamarckian GA in place on `genes` (CUDA [n_runs * pop_size, stride])."""
+        import torch
+        n, stride = genes.shape
+        dev = genes.device
+        E = torch.empty(n, dtype=torch.float32, device=dev)
+        rb = torch.empty(n_runs, 1 + stride, dtype=torch.float32, device=dev)
+        ev = torch.empty(n_runs, dtype=torch.int64, device=dev)
+        gn = torch.empty(n_runs, dtype=torch.int32, device=dev)
+        ad_lga_run(self.h, lig_id, n_runs, genes, E, rb, ev, gn,
+                   engine=ENGINES[engine] if isinstance(engine, str) else engine, **kw)
+        return {"energies": E, "run_best": rb, "n_evals": ev, "n_gens": gn}

@@ -82,7 +82,7 @@ struct ad_context {
     // AD_INTRA_MODE=owner|scatter at context creation (tuning knob; scatter measured
     // faster on config 2: 1.40e8 vs 1.26e8 evals/s, profiles/README.md)
     int intra_mode = INTRA_SCATTER;
-    int32_t last_grid = 0, last_block = 0, last_smem = 0;
+    int32_t last_grid = 0, last_block = 0, last_smem = 0, last_maxreg = 0;
     // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
     int32_t pairs_smem_max = 16384;
 };
@@ -1235,14 +1235,22 @@ int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig) {
 // --------------------------------------------------------------- launches
 namespace {
 
-typedef void (*WarpKernel)(const KParams);
+typedef void (*WarpKernelFn)(const KParams);
+struct WarpKernel {
+    WarpKernelFn lo, hi;  // register budgets AD_WARP_MAXNREG / AD_WARP_MAXNREG_HI
+};
+
+template <int E, bool GR, bool LS>
+WarpKernel wk() {
+    return WarpKernel{k_warp_engine<E, GR, LS, AD_WARP_MAXNREG>, k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI>};
+}
 
 WarpKernel pick_warp_kernel(int engine, bool grad, bool ls) {
-    if (ls) return engine == AD_ENGINE_TC        ? k_warp_engine<1, true, true>
-                   : engine == AD_ENGINE_TC_FP16 ? k_warp_engine<2, true, true>
-                                                 : k_warp_engine<0, true, true>;
-    if (!grad) return k_warp_engine<0, false, false>;
-    return engine == AD_ENGINE_TC ? k_warp_engine<1, true, false> : k_warp_engine<0, true, false>;
+    if (ls) return engine == AD_ENGINE_TC        ? wk<1, true, true>()
+                   : engine == AD_ENGINE_TC_FP16 ? wk<2, true, true>()
+                                                 : wk<0, true, true>();
+    if (!grad) return wk<0, false, false>();
+    return engine == AD_ENGINE_TC ? wk<1, true, false>() : wk<0, true, false>();
 }
 
 int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const void* genes, int32_t stride) {
@@ -1279,28 +1287,38 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // Every pose costs the same, so the launch is scored by (fewest waves of CTAs,
     // then most resident warps per SM, then fewest warps per CTA).  Mixed-ligand
     // launches keep power-of-two CTA sizes (pose_ligand groups must stay aligned).
+    // The 128-register variant wins ties (fewer instructions, no spills): it is
+    // chosen whenever it reaches the same waves and resident warps, i.e. when
+    // shared memory, not the register file, bounds the occupancy.
     int best_w = 0, best_active = -1, best_waves = 1 << 30;
     size_t best_smem = 0;
-    for (int w = 1; w <= 16; ++w) {
-        if (req_warps > 0 && w != req_warps) continue;
-        if (p.pose_ligand && (w & (w - 1))) continue;
-        const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
-        if (smem > (size_t)ctx->max_smem_optin) continue;
-        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        int blocks = 0;
-        CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, kern, w * 32, smem));
-        if (blocks <= 0) continue;
-        const int active = blocks * w;
-        const long ctas = (p.n_poses + w - 1) / w;
-        const int waves = (int)((ctas + (long)blocks * ctx->n_sms - 1) / ((long)blocks * ctx->n_sms));
-        if (getenv("AD_DEBUG_LAUNCH"))
-            fprintf(stderr, "[libad] w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld waves=%d\n", w, smem, blocks,
-                    active, ctas, waves);
-        if (waves < best_waves || (waves == best_waves && active > best_active)) {
-            best_waves = waves;
-            best_active = active;
-            best_w = w;
-            best_smem = smem;
+    WarpKernelFn best_k = nullptr;
+    static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
+    for (int v = 1; v >= 0; --v) {
+        const WarpKernelFn k = v ? kern.hi : kern.lo;
+        if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
+        for (int w = 1; w <= 16; ++w) {
+            if (req_warps > 0 && w != req_warps) continue;
+            if (p.pose_ligand && (w & (w - 1))) continue;
+            const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
+            if (smem > (size_t)ctx->max_smem_optin) continue;
+            CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            int blocks = 0;
+            CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, k, w * 32, smem));
+            if (blocks <= 0) continue;
+            const int active = blocks * w;
+            const long ctas = (p.n_poses + w - 1) / w;
+            const int waves = (int)((ctas + (long)blocks * ctx->n_sms - 1) / ((long)blocks * ctx->n_sms));
+            if (getenv("AD_DEBUG_LAUNCH"))
+                fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld waves=%d\n",
+                        v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, waves);
+            if (waves < best_waves || (waves == best_waves && active > best_active)) {
+                best_waves = waves;
+                best_active = active;
+                best_w = w;
+                best_smem = smem;
+                best_k = k;
+            }
         }
     }
     if (best_w == 0 || best_active <= 0)
@@ -1309,7 +1327,8 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     p.smem_blob = L.blob_bytes;
     p.smem_scratch = L.scratch_bytes;
     const int grid = (p.n_poses + best_w - 1) / best_w;
-    kern<<<grid, best_w * 32, best_smem, st>>>(p);
+    best_k<<<grid, best_w * 32, best_smem, st>>>(p);
+    ctx->last_maxreg = best_k == kern.hi ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG;
     ctx->last_grid = grid;
     ctx->last_block = best_w * 32;
     ctx->last_smem = (int32_t)best_smem;
@@ -1426,6 +1445,135 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     return AD_OK;
 }
 
+int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* genes, int32_t geno_stride,
+                   float* energies, float* run_best, int64_t* n_evals, int32_t* n_gens, const ad_lga_params* prm,
+                   void* stream) {
+    if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
+    const int pop = prm->pop_size;
+    if (n_runs < 0 || pop < 2 || pop > 4096) return fail(AD_ERR_INVALID_ARG, "need n_runs >= 0, 2 <= pop_size <= 4096");
+    const int64_t n_ind64 = (int64_t)n_runs * pop;
+    if (n_ind64 > (1 << 30)) return fail(AD_ERR_LIMIT, "population too large");
+    const int n_ind = (int)n_ind64;
+    if (int32_t rc = common_checks(ctx, lig, n_ind, genes, geno_stride)) return rc;
+    if (n_ind > 0 && !energies) return fail(AD_ERR_INVALID_ARG, "energies is NULL");
+    const ad_ls_params& ls = prm->ls;
+    if (ls.engine != AD_ENGINE_SIMT && ls.engine != AD_ENGINE_TC && ls.engine != AD_ENGINE_TC_FP16)
+        return fail(AD_ERR_INVALID_ARG, "LGA runs the warp engines (SIMT, TC, TC_FP16)");
+    if (ls.max_iters < 1 || !(ls.rho >= 0.f && ls.rho < 1.f) || !(ls.eps > 0.f))
+        return fail(AD_ERR_INVALID_ARG, "bad LS parameters");
+    if (ls.warps_per_cta < 0 || ls.warps_per_cta > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta not in 0..16");
+    if (prm->elitism < 0 || prm->elitism > pop || prm->max_gens < 0 || prm->max_evals < 0)
+        return fail(AD_ERR_INVALID_ARG, "bad GA parameters");
+    if (int32_t rc = set_device(ctx)) return rc;
+    if (int32_t rc = check_device_err(ctx)) return rc;
+    if (n_ind == 0) return AD_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    const LigSlot& L = ctx->ligs[lig];
+    const int S = geno_stride;
+    GaParams G{pop, 6 + L.n_tors, S, prm->elitism, prm->cross_rate, prm->mut_rate, prm->tour_rate, prm->ls_rate,
+               prm->dmov, prm->dang, prm->seed};
+    // scratch: next population, LS list + genes + energies, per-run counters
+    float *d_next = nullptr, *d_lsg = nullptr, *d_lse = nullptr;
+    int32_t *d_list = nullptr, *d_cnt = nullptr, *d_per = nullptr, *d_done = nullptr, *d_gens = nullptr,
+            *d_ndone = nullptr;
+    int64_t* d_evals = nullptr;
+    auto cleanup = [&]() {
+        cudaFree(d_next); cudaFree(d_lsg); cudaFree(d_lse); cudaFree(d_list); cudaFree(d_cnt);
+        cudaFree(d_per); cudaFree(d_done); cudaFree(d_gens); cudaFree(d_ndone); cudaFree(d_evals);
+    };
+#define LGA_TRY(expr)                                                                     \
+    do {                                                                                  \
+        cudaError_t e_ = (expr);                                                          \
+        if (e_ != cudaSuccess) {                                                          \
+            cleanup();                                                                    \
+            return fail(e_ == cudaErrorMemoryAllocation ? AD_ERR_OOM : AD_ERR_CUDA, "%s: %s", #expr, \
+                        cudaGetErrorString(e_));                                          \
+        }                                                                                 \
+    } while (0)
+    const size_t rows = (size_t)n_ind * S * sizeof(float);
+    LGA_TRY(cudaMalloc(&d_next, rows));
+    LGA_TRY(cudaMalloc(&d_lsg, rows));
+    LGA_TRY(cudaMalloc(&d_lse, sizeof(float) * n_ind));
+    LGA_TRY(cudaMalloc(&d_list, sizeof(int32_t) * n_ind));
+    LGA_TRY(cudaMalloc(&d_cnt, sizeof(int32_t)));
+    LGA_TRY(cudaMalloc(&d_per, sizeof(int32_t) * n_runs));
+    LGA_TRY(cudaMalloc(&d_done, sizeof(int32_t) * n_runs));
+    LGA_TRY(cudaMalloc(&d_gens, sizeof(int32_t) * n_runs));
+    LGA_TRY(cudaMalloc(&d_ndone, sizeof(int32_t)));
+    LGA_TRY(cudaMalloc(&d_evals, sizeof(int64_t) * n_runs));
+    LGA_TRY(cudaMemsetAsync(d_cnt, 0, sizeof(int32_t), st));
+    LGA_TRY(cudaMemsetAsync(d_per, 0, sizeof(int32_t) * n_runs, st));
+    LGA_TRY(cudaMemsetAsync(d_done, 0, sizeof(int32_t) * n_runs, st));
+    LGA_TRY(cudaMemsetAsync(d_gens, 0, sizeof(int32_t) * n_runs, st));
+    LGA_TRY(cudaMemsetAsync(d_ndone, 0, sizeof(int32_t), st));
+    // evaluations of the initial population: pop per run
+    {
+        std::vector<int64_t> e0(n_runs, (int64_t)pop);
+        LGA_TRY(cudaMemcpyAsync(d_evals, e0.data(), sizeof(int64_t) * n_runs, cudaMemcpyHostToDevice, st));
+        LGA_TRY(cudaStreamSynchronize(st));
+    }
+    auto score_all = [&](float* g) -> int32_t {
+        KParams p = base_params(ctx, lig, nullptr, n_ind, S);
+        p.genes = g;
+        p.energy = energies;
+        return launch_warp(ctx, L, pick_warp_kernel(AD_ENGINE_SIMT, false, false), p, 0, st, false);
+    };
+    if (int32_t rc = score_all(genes)) { cleanup(); return rc; }
+    KParams lp = base_params(ctx, lig, nullptr, n_ind, S);
+    lp.genes = d_lsg;
+    lp.energy = d_lse;
+    lp.max_iters = ls.max_iters;
+    lp.rho = ls.rho;
+    lp.eps = ls.eps;
+    lp.n_active = d_cnt;
+    const bool tc = ls.engine != AD_ENGINE_SIMT;
+    WarpKernel ls_kern = pick_warp_kernel(ls.engine, true, true);
+    // a run that starts finished (budget already spent) takes no generation
+    const bool start_done = prm->max_gens == 0 || (int64_t)pop >= prm->max_evals;
+    int gen = 0;
+    if (start_done) {
+        std::vector<int32_t> ones(n_runs, 1);
+        LGA_TRY(cudaMemcpyAsync(d_done, ones.data(), sizeof(int32_t) * n_runs, cudaMemcpyHostToDevice, st));
+        LGA_TRY(cudaStreamSynchronize(st));
+    }
+    float* cur = genes;
+    float* nxt = d_next;
+    for (; !start_done; ++gen) {
+        // GA(population) -> scores of the new individuals
+        k_ga_generation<<<n_runs, 128, pop, st>>>(G, cur, energies, nxt, d_done, (uint32_t)gen);
+        LGA_TRY(cudaGetLastError());
+        std::swap(cur, nxt);
+        if (int32_t rc = score_all(cur)) { cleanup(); return rc; }
+        // LS(population): compacted list, gather, ADADELTA, scatter back (Lamarckian)
+        k_ga_ls_select<<<n_runs, 128, 0, st>>>(G, d_done, (uint32_t)gen, d_list, d_cnt, d_per);
+        LGA_TRY(cudaGetLastError());
+        const int rb = std::min(65535, (n_ind * S + 255) / 256);
+        k_ga_rows<<<rb, 256, 0, st>>>(d_list, d_cnt, S, cur, d_lsg, false, nullptr, nullptr);
+        LGA_TRY(cudaGetLastError());
+        if (int32_t rc = launch_warp(ctx, L, ls_kern, lp, ls.warps_per_cta, st, tc)) { cleanup(); return rc; }
+        k_ga_rows<<<rb, 256, 0, st>>>(d_list, d_cnt, S, d_lsg, cur, true, d_lse, energies);
+        LGA_TRY(cudaGetLastError());
+        k_ga_update<<<(n_runs + 127) / 128, 128, 0, st>>>(n_runs, pop, ls.max_iters, prm->max_evals, prm->max_gens,
+                                                         d_done, d_evals, d_gens, d_per, d_cnt, d_ndone);
+        LGA_TRY(cudaGetLastError());
+        int32_t h_done = 0;
+        LGA_TRY(cudaMemcpyAsync(&h_done, d_ndone, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+        LGA_TRY(cudaStreamSynchronize(st));
+        if (h_done >= n_runs) break;
+    }
+    if (cur != genes) LGA_TRY(cudaMemcpyAsync(genes, cur, rows, cudaMemcpyDeviceToDevice, st));
+    if (run_best) {
+        k_best_of_run<<<(n_runs + 3) / 4, 128, 0, st>>>(energies, genes, S, G.n_genes, pop, n_runs, run_best);
+        LGA_TRY(cudaGetLastError());
+    }
+    if (n_evals) LGA_TRY(cudaMemcpyAsync(n_evals, d_evals, sizeof(int64_t) * n_runs, cudaMemcpyDeviceToDevice, st));
+    if (n_gens) LGA_TRY(cudaMemcpyAsync(n_gens, d_gens, sizeof(int32_t) * n_runs, cudaMemcpyDeviceToDevice, st));
+    LGA_TRY(cudaStreamSynchronize(st));
+#undef LGA_TRY
+    cleanup();
+    return AD_OK;
+}
+
 int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
                          const float* partials, float* out, void* stream) {
     if (!ctx || !partials || !out) return fail(AD_ERR_INVALID_ARG, "null argument");
@@ -1495,6 +1643,10 @@ int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
         for (int q = 0; q < std::min<int>(cap, (int)s.rec.size()); ++q) out_rec[q] = s.rec[q];
     return AD_OK;
 }
+
+// Host-only inspection hook (not in include/ad.h): register budget of the last
+// warp-engine launch (AD_WARP_MAXNREG or AD_WARP_MAXNREG_HI).
+int32_t adx_last_maxreg(ad_context* ctx) { return ctx ? ctx->last_maxreg : 0; }
 
 int32_t ad_last_launch(ad_context* ctx, int32_t* grid, int32_t* block, int32_t* smem_bytes) {
     if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");

@@ -213,6 +213,14 @@ struct KParams {
     int32_t smem_blob;      // bytes reserved for the blob in shared memory
     int32_t smem_scratch;   // bytes per warp (SIMT/TC) or per block (baseline)
     int32_t n_ligs;
+    const int32_t* n_active;  // optional device count: poses >= *n_active exit (LGA's compacted LS list)
+};
+
+// NEXT-3 GA generation parameters (ad_lga_params minus the LS part)
+struct GaParams {
+    int32_t pop, n_genes, stride, elitism;
+    float cross_rate, mut_rate, tour_rate, ls_rate, dmov, dang;
+    uint64_t seed;
 };
 
 // device error bits

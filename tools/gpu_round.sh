@@ -1,6 +1,7 @@
 #!/bin/bash
 # One GPU iteration: tests, bench lines, optional ncu captures.
-#   bash tools/gpu_round.sh TAG [tests] [bench] [ncu] [launches]
+#   bash tools/gpu_round.sh TAG [tests] [smoke] [bench] [bench3] [ncu] [ncu_paper] [accuracy] [reduce] [ab] [launches]
+#   (ab: AB_LIBS='lib1.so lib2.so ...' in the environment)
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 TAG=${1:-dev}; shift
 mkdir -p gpurun_out
@@ -28,6 +29,12 @@ for what in "$@"; do
     ncu_paper)
       timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_block_baseline -s 1 -c 1 \
         -o gpurun_out/prof_paper_$TAG python tools/prof_ls.py 2 paper 2 > gpurun_out/ncu_paper_$TAG.log 2>&1 ;;
+    accuracy)
+      timeout 900 python tools/accuracy_study.py gpurun_out/accuracy_$TAG.json > gpurun_out/accuracy_$TAG.log 2>&1; tail -3 gpurun_out/accuracy_$TAG.log ;;
+    reduce)
+      timeout 900 python tools/bench_reduce.py gpurun_out/reduce_$TAG.json 100 > gpurun_out/reduce_$TAG.log 2>&1; tail -25 gpurun_out/reduce_$TAG.log ;;
+    ab)
+      timeout 1200 python tools/ab.py 2 simt $AB_LIBS 2>&1 | tail -8 ;;
     launches)
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$TAG.csv \
         python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/bench_under_ncu_$TAG.log 2>&1 ;;
