@@ -1200,6 +1200,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.stage_bytes = H.pairs_gmem ? H.off_prec : H.blob_bytes;
     const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
     H.scratch_bytes = ws.bytes;
+    H.ws_g = ws.g; H.ws_w = ws.w; H.ws_d = ws.d; H.ws_trig = ws.trig;
+    H.ws_tw = ws.tw; H.ws_genes = ws.genes; H.ws_part = ws.part;
     memcpy(B.buf.data(), &H, sizeof(H));
 
     if (int32_t rc = set_device(ctx)) return rc;
@@ -1240,17 +1242,30 @@ struct WarpKernel {
     WarpKernelFn lo, hi;  // register budgets AD_WARP_MAXNREG / AD_WARP_MAXNREG_HI
 };
 
-template <int E, bool GR, bool LS>
+template <int E, bool GR, bool LS, bool W>
 WarpKernel wk() {
-    return WarpKernel{k_warp_engine<E, GR, LS, AD_WARP_MAXNREG>, k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI>};
+    return WarpKernel{k_warp_engine<E, GR, LS, AD_WARP_MAXNREG, W>, k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W>};
 }
 
-WarpKernel pick_warp_kernel(int engine, bool grad, bool ls) {
-    if (ls) return engine == AD_ENGINE_TC        ? wk<1, true, true>()
-                   : engine == AD_ENGINE_TC_FP16 ? wk<2, true, true>()
-                                                 : wk<0, true, true>();
-    if (!grad) return wk<0, false, false>();
-    return engine == AD_ENGINE_TC ? wk<1, true, false>() : wk<0, true, false>();
+template <bool W>
+WarpKernel pick_warp_kernel_w(int engine, bool grad, bool ls) {
+    if (ls) return engine == AD_ENGINE_TC        ? wk<1, true, true, W>()
+                   : engine == AD_ENGINE_TC_FP16 ? wk<2, true, true, W>()
+                                                 : wk<0, true, true, W>();
+    if (!grad) return wk<0, false, false, W>();
+    return engine == AD_ENGINE_TC ? wk<1, true, false, W>() : wk<0, true, false, W>();
+}
+
+// wide = some ligand the launch may touch has more than 32 genes
+WarpKernel pick_warp_kernel(int engine, bool grad, bool ls, bool wide) {
+    return wide ? pick_warp_kernel_w<true>(engine, grad, ls) : pick_warp_kernel_w<false>(engine, grad, ls);
+}
+
+bool launch_is_wide(const ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand) {
+    if (!pose_ligand) return 6 + ctx->ligs[lig].n_tors > 32;
+    for (const LigSlot& o : ctx->ligs)
+        if (o.live && 6 + o.n_tors > 32) return true;
+    return false;
 }
 
 int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const void* genes, int32_t stride) {
@@ -1372,7 +1387,7 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
     p.grad = grad;
     p.aux = aux;
     const bool want_grad = grad != nullptr || aux != nullptr;
-    return launch_warp(ctx, ctx->ligs[lig], pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false), p, 0,
+    return launch_warp(ctx, ctx->ligs[lig], pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false, launch_is_wide(ctx, lig, pose_ligand)), p, 0,
                        (cudaStream_t)stream, false);
 }
 
@@ -1429,7 +1444,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     } else {
         int w = prm->warps_per_cta;
         if (w < 0 || w > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..16", w);
-        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true), p, w, st,
+        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true, launch_is_wide(ctx, lig, pose_ligand)), p, w, st,
                                      prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16))
             return rc;
     }
@@ -1516,7 +1531,7 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
         KParams p = base_params(ctx, lig, nullptr, n_ind, S);
         p.genes = g;
         p.energy = energies;
-        return launch_warp(ctx, L, pick_warp_kernel(AD_ENGINE_SIMT, false, false), p, 0, st, false);
+        return launch_warp(ctx, L, pick_warp_kernel(AD_ENGINE_SIMT, false, false, launch_is_wide(ctx, lig, nullptr)), p, 0, st, false);
     };
     if (int32_t rc = score_all(genes)) { cleanup(); return rc; }
     KParams lp = base_params(ctx, lig, nullptr, n_ind, S);
@@ -1527,7 +1542,7 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
     lp.eps = ls.eps;
     lp.n_active = d_cnt;
     const bool tc = ls.engine != AD_ENGINE_SIMT;
-    WarpKernel ls_kern = pick_warp_kernel(ls.engine, true, true);
+    WarpKernel ls_kern = pick_warp_kernel(ls.engine, true, true, launch_is_wide(ctx, lig, nullptr));
     // a run that starts finished (budget already spent) takes no generation
     const bool start_done = prm->max_gens == 0 || (int64_t)pop >= prm->max_evals;
     int gen = 0;

@@ -4,7 +4,7 @@
 // shared memory with a single TMA bulk copy (cp.async.bulk) and keeps for all
 // max_iters ADADELTA iterations.  Layout (offsets in LigHeader, bytes):
 //
-//   LigHeader                                   176 B
+//   LigHeader                                   208 B
 //   atoms   float4 [N]      reference x,y,z (A, DFS order), charge q
 //   info    int2   [N]      {map | type<<8 | chain_len<<16 | slot<<24, chain_start}; slot =
 //                           the atom's storage row in the per-pose X / gradient arrays
@@ -74,10 +74,12 @@ struct alignas(16) LigHeader {
     int32_t off_chain, off_mask, off_prec, off_pdsv;    // 64
     int32_t off_tp, scratch_bytes, n_pad, intra_mode;   // 80
     int32_t n_entries, n_chunks, off_comb, off_combidx; // 96  (owner mode: E per lane, chunks per lane)
-    int32_t pairs_gmem, stage_bytes, reserved0, reserved1;  // 112: schedule in global memory?, bytes staged to smem
-    float ff[FF_N];                                     // 176
+    int32_t pairs_gmem, stage_bytes, ws_g, ws_w;        // 112: schedule in global memory?, bytes staged to smem
+    int32_t ws_d, ws_trig, ws_tw, ws_genes;             // 128  per-warp scratch offsets (WarpScratch, ws_x = 0),
+    int32_t ws_part, reserved0, reserved1, reserved2;   // 144  precomputed so kernels reload, not recompute, them
+    float ff[FF_N];                                     // 208
 };
-static_assert(sizeof(LigHeader) == 176, "header size");
+static_assert(sizeof(LigHeader) == 208, "header size");
 
 // Device table entry, one per uploaded ligand.
 struct LigDev {
