@@ -141,7 +141,7 @@ struct BlobBuilder {
 struct Schedule {
     int rounds = 0, slots = 1;
     std::vector<uint32_t> rec;  // [rounds*32]
-    std::vector<float> dsv;     // [rounds*32]
+    std::vector<float> dsv;     // scatter: [rounds*64][2] (dsv, cqq); owner / hybrid: [entries] dsv
 };
 
 // Swap the roles of i and j in a schedule record (the pair term is symmetric;
@@ -541,8 +541,10 @@ int rebalance_steps(std::vector<std::vector<int>>& steps, const std::vector<int>
     return total;
 }
 
+// pdsv / pcq: per pair desolvation prefactor and coeff_el q_i q_j; the schedule
+// stores them interleaved (float2 per entry; empty places (0, 0))
 Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
-                        const std::vector<int>& ptp, const std::vector<float>& pdsv) {
+                        const std::vector<int>& ptp, const std::vector<float>& pdsv, const std::vector<float>& pcq) {
     const int P = (int)pi.size();
     const int target = (P + kPairsPerStep - 1) / kPairsPerStep;
     Schedule best;
@@ -622,7 +624,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
     }
     // entry l of step r goes to lane l % 32, sub-step l / 32: index (2r + l/32)*32 + l%32 = 64r + l
     best.rec.assign((size_t)best_rounds.size() * kPairsPerStep, 0u);
-    best.dsv.assign((size_t)best_rounds.size() * kPairsPerStep, 0.f);
+    best.dsv.assign((size_t)best_rounds.size() * kPairsPerStep * 2, 0.f);
     // steps are arranged independently (deterministic per step): spread them over
     // the host's cores
     std::atomic<size_t> next{0};
@@ -631,7 +633,8 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
             const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots);
             for (int l = 0; l < kPairsPerStep; ++l) {
                 best.rec[r * kPairsPerStep + l] = lay[l].second;
-                best.dsv[r * kPairsPerStep + l] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
+                best.dsv[2 * (r * kPairsPerStep + l)] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
+                best.dsv[2 * (r * kPairsPerStep + l) + 1] = lay[l].first < 0 ? 0.f : pcq[lay[l].first];
             }
         }
     };
@@ -1069,7 +1072,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     const ad_ff_params& F = *d->ff;
     // --- pairs (new numbering) with desolvation prefactors
     std::vector<int> pi(P), pj(P), ptp(P);
-    std::vector<float> pd(P);
+    std::vector<float> pd(P), pcq(P);
     for (int q = 0; q < P; ++q) {
         const int i = d->pairs[2 * q], j = d->pairs[2 * q + 1];
         if (i < 0 || i >= N || j < 0 || j >= N || i == j) return fail(AD_ERR_INVALID_ARG, "pair %d = (%d,%d) invalid", q, i, j);
@@ -1080,6 +1083,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         const double qi = std::fabs((double)d->charge[i]), qj = std::fabs((double)d->charge[j]);
         pd[q] = (float)((double)F.coeff_ds * (((double)d->type_S[ti] + (double)F.qasp * qi) * (double)d->type_V[tj] +
                                               ((double)d->type_S[tj] + (double)F.qasp * qj) * (double)d->type_V[ti]));
+        pcq[q] = (float)((double)F.coeff_el * (double)d->charge[i] * (double)d->charge[j]);
     }
     if (nt * nt > 256) return fail(AD_ERR_LIMIT, "n_types^2 > 256");
     const int mode = ctx->intra_mode;
@@ -1111,7 +1115,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             si[q] = slot[pi[q]];
             sj[q] = slot[pj[q]];
         }
-        sch = schedule_pairs(N, si, sj, ptp, pd);
+        sch = schedule_pairs(N, si, sj, ptp, pd, pcq);
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -1651,7 +1655,7 @@ int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
     }
     if (out_atom_slot)
         for (int a = 0; a < n_atoms; ++a) out_atom_slot[a] = slot[a];
-    const Schedule s = schedule_pairs(n_atoms, pi, pj, ptp, pd);
+    const Schedule s = schedule_pairs(n_atoms, pi, pj, ptp, pd, pd);
     *out_steps = s.rounds;
     *out_slots = s.slots;
     if (out_rec)

@@ -17,7 +17,8 @@
 //                           (slot_i == K marks an empty place).  Step r holds entries
 //                           [64r, 64r+64): lane l takes 64r+l and 64r+32+l; within a
 //                           step every (slot, atom) target is distinct -> no atomics.
-//   pdsv    f32    [R*64]   per pair desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi]
+//   pdsv    f32x2  [R*64]   per pair (desolvation prefactor c_ds[(Si+Q|qi|)Vj+(Sj+Q|qj|)Vi],
+//                           coeff_el q_i q_j), both rounded once from FP64
 //           (INTRA_OWNER: prec/pdsv hold [E][32] directed entries a|b<<8|tp<<16|flags<<24
 //            instead, plus comb int2 [N] (start, count) into combidx u16 [..] = the
 //            partial slots k*32+lane that belong to atom a)
@@ -111,7 +112,7 @@ struct GridDev {
 // Per-warp scratch layout (offsets in bytes from the warp's slice; 16-aligned).
 struct WarpScratch {
     int32_t x;      // float4 [Npad]        world coords + charge
-    int32_t g;      // float4 [K][Npad]     atom gradient accumulators (slot 0 seeded with inter)
+    int32_t g;      // float4 [K][Npad]+8   atom gradient accumulators (slot 0 seeded with inter) + 8 spare
     int32_t w;      // float4 [Npad+1][2]   prefix sums (SIMT) / W staging (TC)
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
     int32_t trig;   // float2 [T]           cos, sin of torsion angles
@@ -131,9 +132,9 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
     int32_t o = 0;
     s.x = o;     o += 16 * npad;
-    // rows of npad float4 (slot k of atom a at k * npad + a) + a spare row targeted
-    // by empty schedule places
-    s.g = o;     o += 16 * npad * (n_slots + 1);
+    // rows of npad float4 (slot k of atom a at k * npad + a) + the start of a spare
+    // row K: empty schedule places only ever target K * npad + (0..7)
+    s.g = o;     o += 16 * npad * n_slots + 16 * 8;
     s.w = o;     o += 32 * (npad + 1);
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);

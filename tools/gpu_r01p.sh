@@ -1,4 +1,4 @@
 cd $GRAFT_REPO_ROOT
 timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider > gpurun_out/pytest_r01p.log 2>&1; tail -2 gpurun_out/pytest_r01p.log; grep -E "^FAILED" gpurun_out/pytest_r01p.log | head
-bash tools/gpu_ab.sh 2 simt build/ab/libad_wd.so build/ab/libad_ir.so
-bash tools/gpu_ab.sh 3 simt build/ab/libad_wd.so build/ab/libad_ir.so
+bash tools/gpu_ab.sh 2 simt build/ab/libad_ir.so build/ab/libad_cq.so
+bash tools/gpu_ab.sh 3 simt build/ab/libad_ir.so build/ab/libad_cq.so
