@@ -1306,14 +1306,16 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // Every pose costs the same, so the launch is scored by (fewest waves of CTAs,
     // then most resident warps per SM, then fewest warps per CTA).  Mixed-ligand
     // launches keep power-of-two CTA sizes (pose_ligand groups must stay aligned).
-    // The 128-register variant wins ties (fewer instructions, no spills): it is
-    // chosen whenever it reaches the same waves and resident warps, i.e. when
-    // shared memory, not the register file, bounds the occupancy.
-    int best_w = 0, best_active = -1, best_waves = 1 << 30;
-    size_t best_smem = 0;
-    WarpKernelFn best_k = nullptr;
+    // Per variant, the best W: fewest waves of CTAs, then most resident warps.
+    // Between the variants: the 128-register twin executes ~10 % fewer instructions
+    // and no spills, which outweighs a few more waves of a long launch (config 3:
+    // 7 waves at 16 warps/SM, 128.3 ms, beat 6 waves at 18, 147.7 ms); the
+    // 80-register twin wins only when its extra occupancy fits a short launch into
+    // fewer waves, at most 2 (config 2: 1 wave at 24 warps/SM vs 2 waves).
+    struct Cand { int w = 0, active = -1, waves = 1 << 30; size_t smem = 0; WarpKernelFn k = nullptr; };
+    Cand cand[2];
     static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
-    for (int v = 1; v >= 0; --v) {
+    for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
         if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
         for (int w = 1; w <= 16; ++w) {
@@ -1331,15 +1333,16 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             if (getenv("AD_DEBUG_LAUNCH"))
                 fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld waves=%d\n",
                         v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, waves);
-            if (waves < best_waves || (waves == best_waves && active > best_active)) {
-                best_waves = waves;
-                best_active = active;
-                best_w = w;
-                best_smem = smem;
-                best_k = k;
-            }
+            Cand& c = cand[v];
+            if (waves < c.waves || (waves == c.waves && active > c.active)) c = Cand{w, active, waves, smem, k};
         }
     }
+    const bool lo_ok = cand[0].k != nullptr, hi_ok = cand[1].k != nullptr;
+    const bool use_lo = lo_ok && (!hi_ok || (cand[0].waves < cand[1].waves && cand[0].waves <= 2));
+    const Cand& pick = use_lo ? cand[0] : cand[1];
+    const int best_w = pick.w, best_active = pick.active;
+    const size_t best_smem = pick.smem;
+    const WarpKernelFn best_k = pick.k;
     if (best_w == 0 || best_active <= 0)
         return fail(AD_ERR_LIMIT, "ligand footprint (%d B blob + %d B/warp) does not fit shared memory", L.blob_bytes,
                     L.scratch_bytes);
