@@ -355,3 +355,29 @@ def test_local_search_fp16_engine(ctx, cfg2):
         rel[eng] = np.linalg.norm(g - Go[:, :Gn], axis=1) / np.maximum(np.linalg.norm(Go[:, :Gn], axis=1), 1e-6)
     assert np.median(rel["tc_fp16"]) > 10 * np.median(rel["tc"])
     assert np.median(rel["tc_fp16"]) < 0.05
+
+
+@pytest.mark.parametrize("mode", ["owner", "hybrid"])
+def test_alternative_intra_modes(ad, cfg2, mode, monkeypatch):
+    """The two non-default pair-loop designs (AD_INTRA_MODE, read at context
+    creation): same parity gates as the default scatter schedule, and
+    the same LS trajectories to FP32 accuracy on the first steps."""
+    monkeypatch.setenv("AD_INTRA_MODE", mode)
+    c = ad.Context(0)
+    try:
+        w = cfg2
+        c.upload_grid(w.grid)
+        lid = c.upload_ligand(w.ligands[0], w.ff)
+        n = 128
+        g = torch.from_numpy(w.genes[:n]).cuda()
+        E, G, _ = c.score(lid, g, grad=True)
+        torch.cuda.synchronize()
+        check_scores(w.ligands[0], w.grid, w.ff, w.genes[:n], E.cpu().numpy(), G.cpu().numpy(), f"cfg2 {mode}")
+        tr, _, _, nev, _ = _ls(c, lid, w.genes[:16], "simt", 20)
+        assert nev == 16 * 20
+        stride = w.genes.shape[1]
+        flat = tr.reshape(16 * 20, -1)
+        check_scores(w.ligands[0], w.grid, w.ff, flat[::7, 1:1 + stride], flat[::7, 0], flat[::7, 1 + stride:],
+                     f"cfg2 {mode} LS")
+    finally:
+        c.close()
