@@ -1303,17 +1303,20 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
                 L.scratch_bytes = std::max(L.scratch_bytes, tc_engine ? o.scratch_bytes : o.scratch_simt);
             }
     }
-    // Every pose costs the same, so the launch is scored by (fewest waves of CTAs,
-    // then most resident warps per SM, then fewest warps per CTA).  Mixed-ligand
-    // launches keep power-of-two CTA sizes (pose_ligand groups must stay aligned).
-    // Per variant, the best W: fewest waves of CTAs, then most resident warps.
-    // Between the variants: the 128-register twin executes ~10 % fewer instructions
-    // and no spills, which outweighs a few more waves of a long launch (config 3:
-    // 7 waves at 16 warps/SM, 128.3 ms, beat 6 waves at 18, 147.7 ms); the
-    // 80-register twin wins only when its extra occupancy fits a short launch into
-    // fewer waves, at most 2 (config 2: 1 wave at 24 warps/SM vs 2 waves).
-    struct Cand { int w = 0, active = -1, waves = 1 << 30; size_t smem = 0; WarpKernelFn k = nullptr; };
-    Cand cand[2];
+    // Every pose costs the same.  A launch shape (register variant, W warps per CTA)
+    // is scored by the modelled time of the busiest SM: it receives ceil(CTAs / SMs)
+    // CTAs and runs them in waves of `blocks` resident CTAs; a wave of a warps
+    // (a poses) takes a^(1 - gamma) time units, i.e. per-SM throughput grows as
+    // a^gamma with the resident warps (partial latency hiding).  gamma = 0.48 fits
+    // the measured config-2 shapes (tools/ab.py, ms per LS launch): W = 6 (4 CTAs =
+    // 24 poses on the busiest SM) 4.14, W = 7 (3 CTAs = 21 poses) 3.87, W = 11
+    // (22 poses) 3.87, W = 8 (24 poses) 4.02.  The 128-register twin executes
+    // ~10 % fewer instructions and no spills: its time is scaled by 0.85 (config 3,
+    // smem-bound at 16 warps/SM either way: 128.3 ms vs 147.7 ms for the 80-register
+    // twin at 18).  Ties: more resident warps, then fewer CTAs (fewer blob stagings).
+    // Mixed-ligand launches keep power-of-two CTA sizes (pose_ligand groups stay aligned).
+    struct Cand { int w = 0, active = -1; double cost = 1e300; long ctas = 0; size_t smem = 0; WarpKernelFn k = nullptr; };
+    Cand pick;
     static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
     for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
@@ -1329,17 +1332,19 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             if (blocks <= 0) continue;
             const int active = blocks * w;
             const long ctas = (p.n_poses + w - 1) / w;
-            const int waves = (int)((ctas + (long)blocks * ctx->n_sms - 1) / ((long)blocks * ctx->n_sms));
+            const long per_sm = (ctas + ctx->n_sms - 1) / ctx->n_sms;  // CTAs on the busiest SM
+            const long full = per_sm / blocks, rem = per_sm % blocks;
+            const double g1 = 1.0 - 0.48;
+            double cost = (double)full * std::pow((double)active, g1) + (rem ? std::pow((double)(rem * w), g1) : 0.0);
+            if (v) cost *= 0.85;
             if (getenv("AD_DEBUG_LAUNCH"))
-                fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld waves=%d\n",
-                        v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, waves);
-            Cand& c = cand[v];
-            if (waves < c.waves || (waves == c.waves && active > c.active)) c = Cand{w, active, waves, smem, k};
+                fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld per_sm=%ld cost=%.3f\n",
+                        v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, per_sm, cost);
+            const bool better = cost < pick.cost - 1e-9 ||
+                                (cost < pick.cost + 1e-9 && (active > pick.active || (active == pick.active && ctas < pick.ctas)));
+            if (better) pick = Cand{w, active, cost, ctas, smem, k};
         }
     }
-    const bool lo_ok = cand[0].k != nullptr, hi_ok = cand[1].k != nullptr;
-    const bool use_lo = lo_ok && (!hi_ok || (cand[0].waves < cand[1].waves && cand[0].waves <= 2));
-    const Cand& pick = use_lo ? cand[0] : cand[1];
     const int best_w = pick.w, best_active = pick.active;
     const size_t best_smem = pick.smem;
     const WarpKernelFn best_k = pick.k;

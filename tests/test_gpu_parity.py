@@ -170,25 +170,33 @@ def test_engines_agree_on_first_steps(ctx, cfg2):
         assert np.all(d <= 1e-5 * np.abs(trs["simt"][:, 0, 0]) + 1e-3)
 
 
-def test_full_size_sampled(ctx, cfg2):
-    """BASELINE config 2 at full size (3000 poses x 300 iterations) in the bench
-    launch configuration (TC engine, library-chosen CTA shape): properties on all
-    poses, oracle parity on sampled evaluations."""
-    (lid,) = _setup(ctx, cfg2, "cfg2")
-    L = cfg2.ligands[0]
-    Gn = L.n_genes
-    stride = cfg2.genes.shape[1]
-    tr, bE, best_genes, nev, _ = _ls(ctx, lid, cfg2.genes, "tc", 300, pop_per_run=150)
-    n = cfg2.n_poses
-    assert nev == n * 300
-    assert np.array_equal(bE, tr[:, :, 0].min(axis=1))
-    assert np.all(np.isfinite(bE))
-    rng = np.random.default_rng(1)
-    sel = rng.choice(n * 300, size=96, replace=False)
-    flat = tr.reshape(n * 300, -1)
-    check_scores(L, cfg2.grid, cfg2.ff, flat[sel, 1:1 + stride], flat[sel, 0], flat[sel, 1 + stride:], "cfg2 full")
+@pytest.mark.parametrize("which,engine", [("cfg2", "simt"), ("cfg2", "tc"), ("cfg3", "simt")])
+def test_full_size_sampled(ctx, which, engine, request):
+    """BASELINE configs 2 and 3 at full size (3000 / 15000 poses x 300 iterations) in
+    the bench launch configuration (library-chosen CTA shape and register variant;
+    simt = the bench default engine): properties on all poses (on the device),
+    oracle parity on sampled evaluations of the trace."""
+    w = request.getfixturevalue(which)
+    (lid,) = _setup(ctx, w, which)
+    L = w.ligands[0]
+    stride = w.genes.shape[1]
+    n, iters = w.n_poses, w.iters
+    g = torch.from_numpy(w.genes).cuda()
+    nev = torch.zeros(1, dtype=torch.int64, device="cuda")
+    out = ctx.local_search(lid, g, max_iters=iters, engine=engine, trace=True, n_evals=nev, pop_per_run=w.pop)
+    torch.cuda.synchronize()
+    tr = out["trace"].view(n, iters, -1)
+    bE = out["best_energy"]
+    assert int(nev.item()) == n * iters
+    assert torch.equal(bE, tr[:, :, 0].min(dim=1).values)
+    assert bool(torch.isfinite(bE).all())
     # the search makes progress: best energy well below the start energy for most poses
-    assert np.mean(bE < tr[:, 0, 0]) > 0.9
+    assert float((bE < tr[:, 0, 0]).float().mean()) > 0.9
+    rng = np.random.default_rng(1)
+    sel = torch.from_numpy(rng.choice(n * iters, size=96, replace=False)).cuda()
+    flat = tr.reshape(n * iters, -1)[sel].cpu().numpy()
+    del out, tr
+    check_scores(L, w.grid, w.ff, flat[:, 1:1 + stride], flat[:, 0], flat[:, 1 + stride:], f"{which} full {engine}")
 
 
 def test_edge_cases(ctx, ad):

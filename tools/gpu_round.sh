@@ -37,7 +37,7 @@ for what in "$@"; do
       timeout 1200 python tools/ab.py 2 simt $AB_LIBS 2>&1 | tail -8 ;;
     launches)
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$TAG.csv \
-        python bench.py --steps 2 --warmup 1 --no-cpu-baseline > gpurun_out/bench_under_ncu_$TAG.log 2>&1 ;;
+        python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-paper-engine > gpurun_out/bench_under_ncu_$TAG.log 2>&1 ;;
   esac
 done
 ls gpurun_out | tail -30
