@@ -495,9 +495,18 @@ int rebalance_steps(std::vector<std::vector<int>>& steps, const std::vector<int>
         }
         total += over(deg[a]);
     }
+    // lower bound: a bank group with more than cap * R ends overall stays overloaded
+    // however the pairs are spread (stop there instead of spending all iterations)
+    int bound = 0;
+    {
+        int g_all[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        for (int a = 0; a < R; ++a)
+            for (int r = 0; r < 8; ++r) g_all[r] += deg[a][r];
+        for (int r = 0; r < 8; ++r) bound += std::max(0, g_all[r] - cap * R);
+    }
     uint64_t st = 0xD1B54A32D192ED03ull;
     auto rnd = [&]() { st ^= st << 13; st ^= st >> 7; st ^= st << 17; return st; };
-    for (long it = 0; it < iters && total > 0; ++it) {
+    for (long it = 0; it < iters && total > bound; ++it) {
         const int A = (int)(rnd() % R), B = (int)(rnd() % R);
         if (A == B || steps[A].empty()) continue;
         if (over(deg[A]) == 0 && over(deg[B]) == 0) continue;
