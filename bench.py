@@ -44,7 +44,11 @@ def parse():
     # only if it wins, north_star); `--engine tc` times the tensor-core engine
     ap.add_argument("--engine", default="simt", choices=["simt", "tc", "tc_fp16", "paper", "paper_tcec"])
     ap.add_argument("--warps", type=int, default=0, help="warps per CTA (0 = library choice)")
-    ap.add_argument("--config", type=int, default=2, choices=[2, 3])
+    ap.add_argument("--config", type=int, default=2, choices=[2, 3, 5])
+    # config 5 (virtual screen, strong scaling over the ranks)
+    ap.add_argument("--ligands", type=int, default=8192, help="config 5: ligands in the screen")
+    ap.add_argument("--effort", type=int, default=1, help="config 5: pair-schedule placement effort (0..2)")
+    ap.add_argument("--buckets", type=int, default=8, help="config 5: launches per rank per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-paper-engine", action="store_true")
     return ap.parse_args()
@@ -162,6 +166,36 @@ def load_traffic(engine, config):
         return None
 
 
+def run_reference_screen(args, O, synth):
+    """--impl reference --config 5: the oracle on a bounded sample of the screen
+    (every step: 1 run x pop poses x 300 iterations of 8 ligands spread over the
+    size draws), evals/s on the host cores."""
+    spec = synth.ScreenSpec(n_ligands=args.ligands)
+    cores = len(os.sched_getaffinity(0))
+    ff = synth.FFParams()
+    ks = sorted(range(spec.n_ligands), key=lambda k: spec.sizes[k])
+    ks = [ks[int(i)] for i in np.linspace(0, len(ks) - 1, 8)]
+    work = [(spec.ligand(k), spec.genes(k)[:spec.pop]) for k in ks]
+    for _ in range(args.warmup):
+        O.local_search(work[0][0], spec.grid, ff, work[0][1], max_iters=spec.iters, threads=cores)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for L, g in work:
+            O.local_search(L, spec.grid, ff, g, max_iters=spec.iters, threads=cores)
+    dt = time.perf_counter() - t0
+    val = args.steps * len(work) * spec.pop * spec.iters / dt
+    sample = (f"1 run x {spec.pop} pop x {spec.iters} ADADELTA iterations of 8 of the {spec.n_ligands} screen "
+              f"ligands ({work[0][0].n_atoms}-{work[-1][0].n_atoms} atoms) per step")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{spec.name}: {spec.n_ligands} ligands x {spec.runs} runs x {spec.pop} pop x "
+                               f"{spec.iters} ADADELTA iterations", "engine": "oracle", "sample": sample},
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
+
+
 def run_reference(args):
     """--impl reference: the FP64 oracle as it stands, on host cores, rank 0 only."""
     rank = int(os.environ.get("RANK", "0"))
@@ -169,6 +203,9 @@ def run_reference(args):
         return
     from oracle import oracle as O
     from paper_conf_sc_solis_vasquezts25_b200 import synth
+    if args.config == 5:
+        run_reference_screen(args, O, synth)
+        return
     w = synth.make_config(args.config)
     lig = w.ligands[0]
     cores = len(os.sched_getaffinity(0))
@@ -194,10 +231,157 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def run_screen_bench(args):
+    """Config 5: the virtual screen (8192 ligands of 20-110 atoms and 0-32 torsions
+    x 20 runs x 16 pop x 300 ADADELTA iterations against the config-2 receptor),
+    (ligand, run) units LPT-sharded over the ranks, one NCCL all_gather of the
+    best-pose records per step.  Strong scaling: the total work is fixed.  One
+    step = every bucket launch of the rank + the gather; ligands are uploaded
+    (and their pair schedules built) once, before the timed region, like the
+    receptor grids."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_solis_vasquezts25_b200 import ad, report, screen, synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    cores = len(os.sched_getaffinity(0))
+    spec = synth.ScreenSpec(n_ligands=args.ligands)
+    ff = synth.FFParams()
+    ctx = ad.Context(local)
+    S = screen.Screen(ctx, spec, ff, rank=rank, world=world, engine=args.engine, n_buckets=args.buckets,
+                      effort=args.effort, upload_threads=max(1, cores // local_world),
+                      gen_processes=max(1, cores // local_world))
+    stream = torch.cuda.current_stream()
+    n_evals = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    for _ in range(args.warmup):
+        S.step()
+    torch.cuda.synchronize()
+    n_evals.zero_()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with ClockSampler(local) as clocks:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        for k in range(args.steps):
+            flush.fill_(float(k))  # L2 flush, outside the timed events
+            ev[k][0].record(stream)
+            rec = S.step(n_evals)
+            ev[k][1].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms = [a.elapsed_time(b) for a, b in ev]
+    total = torch.tensor([sum(ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(total, op=dist.ReduceOp.MAX)
+    total_ms = float(total.item())
+    assert int(n_evals.item()) == args.steps * S.n_poses * spec.iters
+    evals_all = args.steps * spec.n_ligands * spec.runs * spec.pop * spec.iters
+    value = evals_all / (total_ms / 1e3)
+    recs = rec.cpu().numpy()
+    got = recs[~np.isnan(recs[:, 0])]
+    assert len(got) == spec.n_ligands * spec.runs and np.all(np.isfinite(got[:, 2])), "screen records incomplete"
+
+    # end to end: the start genotypes from pinned host memory + the records back, per step
+    h2d = S.pin_host_inputs()
+    h_rec = torch.empty(tuple(rec.shape)).pin_memory()
+    e2e = []
+    for k in range(max(2, args.steps)):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        flush.fill_(float(k))
+        a.record(stream)
+        r = S.step(from_host=True)
+        h_rec.copy_(r, non_blocking=True)
+        b.record(stream)
+        e2e.append((a, b))
+    torch.cuda.synchronize()
+    e2e_t = torch.tensor([sum(a.elapsed_time(b) for a, b in e2e) / len(e2e)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_val = spec.n_ligands * spec.runs * spec.pop * spec.iters / (float(e2e_t.item()) / 1e3)
+
+    # roofline of this rank's LS launches: the flop model per ligand x its evaluations
+    flops = sum(report.ligand_work(S.ligands[k])["flops"] for b in S.buckets for k, _ in b["units"]) * spec.pop * spec.iters
+    achieved = flops / (statistics.mean(ms) / 1e3) / 1e12
+    peak = report.fp32_peak_tflops(1965.0)
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": None, "peak_basis": "148 SMs x 128 FP32 lanes x 2 (FMA) x 1965 MHz max SM clock (DESIGN.md)",
+                "flops_per_step_rank0": flops, "launches_per_step": len(S.buckets)}
+
+    cpu = parity = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        from oracle import oracle as O
+        # the oracle on a bounded sample: the first 2 runs (32 poses, 300 iterations) of 12
+        # ligands spread over the size range; and the GPU's best energies of those units
+        # re-scored by the oracle at the returned genotypes
+        ks = sorted(S.ligands, key=lambda k: S.ligands[k].n_pairs)
+        ks = [ks[int(i)] for i in np.linspace(0, len(ks) - 1, 12)]
+        t0 = time.perf_counter()
+        n_s = 0
+        for k in ks:
+            g = spec.genes(k)[:2 * spec.pop]
+            O.local_search(S.ligands[k], spec.grid, ff, g, max_iters=spec.iters, threads=cores)
+            n_s += len(g) * spec.iters
+        dt = time.perf_counter() - t0
+        cpu = {"value": n_s / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"2 runs x {spec.pop} pop x {spec.iters} ADADELTA iterations of 12 screen ligands "
+                         f"({S.ligands[ks[0]].n_atoms}-{S.ligands[ks[-1]].n_atoms} atoms)"}
+        by_unit = {(int(r[0]), int(r[1])): r for r in got}
+        dE, ok = [], []
+        for k in ks:
+            L = S.ligands[k]
+            for r in range(spec.runs):
+                row = by_unit[(k, r)]
+                Eo, _, aux, _ = O.score(L, spec.grid, ff, row[3:3 + spec.stride][None, :].astype(np.float32))
+                d = abs(float(row[2]) - float(Eo[0]))
+                dE.append(d)
+                ok.append(d <= 1e-3 + 2.0 ** -20 * float(aux[0, O.AUX_ABS_E] + aux[0, O.AUX_SENS_E]))
+        parity = {"max_abs_dE": float(max(dE)), "median_abs_dE": float(np.median(dE)),
+                  "frac_within_gate": float(np.mean(ok)),
+                  "gate": "|dE| <= 1e-3 + 2^-20 (A_E + S_E) (DESIGN.md Tolerances)",
+                  "sample": f"best pose of every run of 12 ligands ({len(dE)} records) re-scored by the FP64 oracle"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{spec.name}: {spec.n_ligands} ligands (20-110 atoms, 0-32 torsions) x "
+                                   f"{spec.runs} runs x {spec.pop} pop x {spec.iters} ADADELTA iterations, 60^3 grid "
+                                   f"x 0.375 A (10 maps), (ligand, run) units LPT-sharded over {world} GPU(s)",
+                       "engine": args.engine, "buckets_per_rank": len(S.buckets), "schedule_effort": args.effort,
+                       "l2": "flushed between timed steps (256 MiB write, outside the timed events)",
+                       "parallelism": f"units sharded, {world} GPU(s), NCCL all_gather of best-pose records",
+                       "setup_s_rank0": S.setup_s},
+            "roofline": roofline, "cpu_baseline": cpu, "parity": parity,
+            "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                    "d2h_bytes_per_step": int(h_rec.numel() * 4)},
+            "clocks": clocks.summary(), "gpu_launches": 2 * len(S.buckets) * args.steps,  # LS + best-of-run
+        }
+        print(json.dumps(line), flush=True)
+    S.close()
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+        return
+    if args.config == 5:
+        run_screen_bench(args)
         return
     import torch
     import torch.distributed as dist

@@ -18,7 +18,11 @@
  *     surfaces as AD_ERR_CUDA on a later call or stream synchronisation.
  *     Device-side argument errors (bad pose_ligand ids) surface as
  *     AD_ERR_INVALID_ARG on the NEXT call on the same context.
- *   - One context per device per host thread (no internal locking).
+ *   - One context per device per host thread, except ad_upload_ligand and
+ *     ad_free_ligand, which may be called concurrently from several host threads
+ *     on one context (the host-side ligand preparation -- torsion tree, pair
+ *     schedule -- runs unlocked, so a screen's uploads overlap; the device-side
+ *     part is serialised internally).
  *   - Units: Angstrom, kcal/mol, elementary charge, degrees (Z11).
  */
 #ifndef AD_H
@@ -150,23 +154,48 @@ typedef struct {
     const ad_ff_params* ff;     /* scoring constants for this ligand */
 } ad_ligand_desc;
 
-/* Upload a ligand; *out receives its id (>= 0).  Requires a grid (atom_map
- * must index a type map).  Errors: AD_ERR_INVALID_ARG (bad index, a not
- * excluded from its moving set, non-laminar moving sets, i == j pair,
- * unsupported exponents), AD_ERR_LIMIT, AD_ERR_STATE (no grid), AD_ERR_OOM. */
+/* Upload a ligand; *out receives its id (>= 0; the lowest id not in use, so ids
+ * of freed ligands are reused).  Requires a grid (atom_map must index a type
+ * map).  Thread-safe with respect to other uploads / frees on the same context.
+ * Errors: AD_ERR_INVALID_ARG (bad index, a not excluded from its moving set,
+ * non-laminar moving sets, i == j pair, unsupported exponents), AD_ERR_LIMIT,
+ * AD_ERR_STATE (no grid), AD_ERR_OOM. */
 int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* desc, ad_ligand_id* out);
 
 /* Free a ligand's device blob (synchronises the device). */
 int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig);
+
+/* Launch set of later pose_ligand launches (ad_score_poses, ad_local_search,
+ * ad_lga_run with pose_ligand != NULL): the ligands they may reference, which
+ * size their shared memory, pick the >32-gene variant and must share one
+ * ad_ff_params.  ids: host [n] live ligand ids, copied; n == 0 restores the
+ * default (every live ligand).  A launch that references a ligand whose
+ * footprint exceeds the set's fails with AD_ERR_INVALID_ARG on the next call
+ * (device-side check).  A virtual screen keeps all its ligands resident and
+ * sets each bucket's ligands before the bucket's launch.
+ * Errors: AD_ERR_INVALID_ARG (an id not live). */
+int32_t ad_set_launch_ligands(ad_context* ctx, const int32_t* ids, int32_t n);
+
+/* Host effort of later uploads' intra-pair schedule placement (DESIGN.md §7,
+ * "Bank-conflict-free placement"): 2 (default) = full search (1-500 ms of host
+ * time per ligand, conflict-free shared-memory accesses); 1 = a tenth of the
+ * local-search iterations; 0 = construction only (no cross-step rebalancing,
+ * no local search; ~1 ms).  Every effort evaluates the same pairs with the same
+ * arithmetic; only the order of the intra-pair partial sums (FP32 rounding, well
+ * inside the parity gates) and the kernel's shared-memory bank conflicts
+ * (speed) change.  Errors: AD_ERR_INVALID_ARG. */
+int32_t ad_set_schedule_effort(ad_context* ctx, int32_t effort);
 
 /* One energy (+ gradient) evaluation per pose: PoseCalculation -> InterGradient
  * -> IntraGradient -> gene-space sums (Alg 4; energy = inter + intra,
  * O-5).  One warp per pose.
  *   lig          ligand of every pose (if pose_ligand == NULL).
  *   pose_ligand  device [n_poses] ligand ids, or NULL.  Shared memory is then
- *                sized for the largest live ligand, and every aligned group of
- *                poses sharing a CTA must use one ligand (groups of 1, 2, 4 or 8
- *                poses; keep runs of one ligand a multiple of 8 poses long).
+ *                sized for the largest ligand of the launch set (every live
+ *                ligand, or the list given to ad_set_launch_ligands), and every
+ *                aligned group of poses sharing a CTA must use one ligand (groups
+ *                of 1, 2, 4 or 8 poses; keep runs of one ligand a multiple of 8
+ *                poses long).
  *   genes        device [n_poses][geno_stride] FP32, geno_stride >= 6 + n_tors:
  *                translation (grid units), phi, theta, alpha, torsions (degrees).
  *   energy       device [n_poses] FP32 out.

@@ -23,8 +23,8 @@ ENGINES = {"simt": AD_ENGINE_SIMT, "tc": AD_ENGINE_TC, "paper": AD_ENGINE_PAPER_
 
 # names exported by include/ad.h (tests check the .so exports all of them)
 EXPORTS = ("ad_last_error", "ad_version", "ad_context_create", "ad_context_destroy", "ad_upload_grids",
-           "ad_upload_ligand", "ad_free_ligand", "ad_score_poses", "ad_local_search", "ad_lga_run", "ad_reduce_blocks",
-           "ad_query", "ad_last_launch")
+           "ad_upload_ligand", "ad_free_ligand", "ad_set_launch_ligands", "ad_set_schedule_effort",
+           "ad_score_poses", "ad_local_search", "ad_lga_run", "ad_reduce_blocks", "ad_query", "ad_last_launch")
 
 
 class AdError(RuntimeError):
@@ -82,6 +82,8 @@ def lib():
             L.ad_upload_grids.argtypes = [P, C.POINTER(GridDesc), P, I32, P]
             L.ad_upload_ligand.argtypes = [P, C.POINTER(LigandDesc), C.POINTER(I32)]
             L.ad_free_ligand.argtypes = [P, I32]
+            L.ad_set_schedule_effort.argtypes = [P, I32]
+            L.ad_set_launch_ligands.argtypes = [P, P, I32]
             L.ad_score_poses.argtypes = [P, I32, P, I32, P, I32, P, P, P, P]
             L.ad_local_search.argtypes = [P, I32, P, I32, P, I32, P, P, P, C.POINTER(LSParams), P]
             L.ad_reduce_blocks.argtypes = [P, I32, I32, I32, I32, P, P, P]
@@ -165,6 +167,15 @@ def ad_upload_ligand(ctx, lig, ff) -> int:
 
 def ad_free_ligand(ctx, lig: int) -> None:
     _check(lib().ad_free_ligand(ctx, lig))
+
+
+def ad_set_launch_ligands(ctx, ids) -> None:
+    a = np.ascontiguousarray(list(ids) if ids is not None else [], dtype=np.int32)
+    _check(lib().ad_set_launch_ligands(ctx, a.ctypes.data_as(C.c_void_p) if a.size else None, int(a.size)))
+
+
+def ad_set_schedule_effort(ctx, effort: int) -> None:
+    _check(lib().ad_set_schedule_effort(ctx, int(effort)))
 
 
 def ad_score_poses(ctx, lig, pose_ligand, genes, energy, grad=None, aux=None, stream=None) -> None:
@@ -254,6 +265,25 @@ class Context:
 
     def upload_ligand(self, lig, ff) -> int:
         return ad_upload_ligand(self.h, lig, ff)
+
+    def upload_ligands(self, ligs, ff, threads: int = 0) -> list:
+        """Upload many ligands from a pool of host threads (ad_upload_ligand is
+        thread-safe on one context and ctypes releases the GIL, so the host-side
+        preparation of the pair schedules overlaps).  Returns the ids in order."""
+        from concurrent.futures import ThreadPoolExecutor
+        import os
+        n = threads or max(1, min(len(ligs), len(os.sched_getaffinity(0))))
+        with ThreadPoolExecutor(n) as ex:
+            return list(ex.map(lambda L: ad_upload_ligand(self.h, L, ff), ligs))
+
+    def free_ligand(self, lig_id: int) -> None:
+        ad_free_ligand(self.h, lig_id)
+
+    def set_launch_ligands(self, ids=None) -> None:
+        ad_set_launch_ligands(self.h, ids)
+
+    def set_schedule_effort(self, effort: int) -> None:
+        ad_set_schedule_effort(self.h, effort)
 
     def score(self, lig_id, genes, grad=True, aux=False, pose_ligand=None):
         import torch

@@ -20,6 +20,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <mutex>
 #include <thread>
 #include <vector>
 
@@ -85,6 +86,14 @@ struct ad_context {
     int32_t last_grid = 0, last_block = 0, last_smem = 0, last_maxreg = 0;
     // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
     int32_t pairs_smem_max = 16384;
+    // host effort spent on the pair schedule's bank-conflict placement (ad_set_schedule_effort)
+    int32_t sched_effort = 2;
+    // ligands that pose_ligand launches may reference (ad_set_launch_ligands; empty = every
+    // live ligand): shared memory, the wide variant and the common-constants check follow it
+    std::vector<int> launch_set;
+    // serialises the device-side part of ad_upload_ligand / ad_free_ligand (the host-side
+    // ligand preparation runs outside it, so uploads from several threads overlap)
+    std::mutex mu;
 };
 
 namespace {
@@ -108,8 +117,16 @@ int32_t check_device_err(ad_context* ctx) {
     return AD_OK;
 }
 
-int32_t sync_ligtab(ad_context* ctx) {
+// Device table of ligands: entry `only` alone when it fits the allocated table
+// (uploads of a large screen stay O(1) each), else the whole table.
+int32_t sync_ligtab(ad_context* ctx, int only = -1) {
     const int n = (int)ctx->ligs.size();
+    if (only >= 0 && only < ctx->ligtab_cap) {
+        const LigSlot& L = ctx->ligs[only];
+        const LigDev e{L.live ? L.d_blob : nullptr, L.blob_bytes, L.scratch_bytes, L.scratch_simt, 0};
+        CUDA_TRY(cudaMemcpy(ctx->d_ligtab + only, &e, sizeof(LigDev), cudaMemcpyHostToDevice));
+        return AD_OK;
+    }
     if (n > ctx->ligtab_cap) {
         int cap = std::max(64, ctx->ligtab_cap * 2);
         while (cap < n) cap *= 2;
@@ -405,11 +422,10 @@ bool arrange_matching(const std::vector<std::pair<int, uint32_t>>& pool, int n_a
 }
 
 std::vector<std::pair<int, uint32_t>> arrange_step(const std::vector<std::pair<int, uint32_t>>& pool, int n_atoms,
-                                                   int K) {
+                                                   int K, int refine_iters) {
     // two candidates, the lower modelled cost wins: the matching construction (exact
     // when the step's residues allow it) and the greedy grouping; both polished by
     // the local search unless already conflict free
-    static const int refine_iters = getenv("AD_REFINE_ITERS") ? atoi(getenv("AD_REFINE_ITERS")) : 20000;
     const int npad = npad_of(n_atoms);
     auto total = [&](const std::vector<std::pair<int, uint32_t>>& o) {
         int c = 0;
@@ -552,8 +568,15 @@ int rebalance_steps(std::vector<std::vector<int>>& steps, const std::vector<int>
 
 // pdsv / pcq: per pair desolvation prefactor and coeff_el q_i q_j; the schedule
 // stores them interleaved (float2 per entry; empty places (0, 0))
+// effort (ad_set_schedule_effort): 2 = full placement search (the default; ~1-500 ms
+// of host time per ligand), 1 = a tenth of the local-search iterations, 0 = no
+// cross-step rebalancing and no local search (matching / greedy construction only).
 Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vector<int>& pj,
-                        const std::vector<int>& ptp, const std::vector<float>& pdsv, const std::vector<float>& pcq) {
+                        const std::vector<int>& ptp, const std::vector<float>& pdsv, const std::vector<float>& pcq,
+                        int effort = 2) {
+    static const int refine_env = getenv("AD_REFINE_ITERS") ? atoi(getenv("AD_REFINE_ITERS")) : -1;
+    const int refine_iters = refine_env >= 0 ? refine_env : effort >= 2 ? 20000 : effort == 1 ? 2000 : 0;
+    const long rebalance_per_step = effort >= 2 ? 200000L : effort == 1 ? 20000L : 0L;
     const int P = (int)pi.size();
     const int target = (P + kPairsPerStep - 1) / kPairsPerStep;
     Schedule best;
@@ -611,12 +634,12 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
         if (R <= target) break;
     }
     (void)target;
-    if (n_atoms >= 8 && !getenv("AD_NO_REBALANCE")) {
+    if (n_atoms >= 8 && rebalance_per_step > 0 && !getenv("AD_NO_REBALANCE")) {
         // cross-step rebalancing, then slots re-assigned by occurrence order
         std::vector<std::vector<int>> ids(best_rounds.size());
         for (size_t r = 0; r < best_rounds.size(); ++r)
             for (const auto& e : best_rounds[r]) ids[r].push_back(e.first);
-        const int left = rebalance_steps(ids, pi, pj, n_idx, best.slots, 200000L * (long)ids.size());
+        const int left = rebalance_steps(ids, pi, pj, n_idx, best.slots, rebalance_per_step * (long)ids.size());
         if (getenv("AD_DEBUG_SCHEDULE")) fprintf(stderr, "[libad] rebalance: overload left %d\n", left);
         std::vector<int> cnt(n_idx);
         for (size_t r = 0; r < ids.size(); ++r) {
@@ -639,7 +662,7 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
     std::atomic<size_t> next{0};
     auto worker = [&]() {
         for (size_t r; (r = next.fetch_add(1)) < best_rounds.size();) {
-            const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots);
+            const std::vector<std::pair<int, uint32_t>> lay = arrange_step(best_rounds[r], n_atoms, best.slots, refine_iters);
             for (int l = 0; l < kPairsPerStep; ++l) {
                 best.rec[r * kPairsPerStep + l] = lay[l].second;
                 best.dsv[2 * (r * kPairsPerStep + l)] = lay[l].first < 0 ? 0.f : pdsv[lay[l].first];
@@ -989,7 +1012,6 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     if (!d->ref_xyz || !d->atom_map || !d->atom_type || !d->charge || !d->tp_coef || !d->type_S || !d->type_V ||
         !d->ff || (T && (!d->tors_axis || !d->tors_moving)) || (P && !d->pairs))
         return fail(AD_ERR_INVALID_ARG, "null array in ligand descriptor");
-    if ((int64_t)ctx->ligs.size() >= AD_MAX_LIGANDS) return fail(AD_ERR_LIMIT, "too many ligands");
     for (int a = 0; a < N; ++a) {
         if (d->atom_map[a] < 0 || d->atom_map[a] >= ctx->grid_n_type)
             return fail(AD_ERR_INVALID_ARG, "atom_map[%d]=%d not a type map", a, d->atom_map[a]);
@@ -1124,7 +1146,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             si[q] = slot[pi[q]];
             sj[q] = slot[pj[q]];
         }
-        sch = schedule_pairs(N, si, sj, ptp, pd, pcq);
+        sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -1217,6 +1239,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.ws_tw = ws.tw; H.ws_genes = ws.genes; H.ws_part = ws.part;
     memcpy(B.buf.data(), &H, sizeof(H));
 
+    std::lock_guard<std::mutex> lock(ctx->mu);
     if (int32_t rc = set_device(ctx)) return rc;
     LigSlot s;
     s.blob_bytes = H.stage_bytes;  // shared-memory bytes staged per CTA
@@ -1229,20 +1252,48 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     CUDA_TRY(cudaMalloc(&s.d_blob, B.buf.size()));
     CUDA_TRY(cudaMemcpy(s.d_blob, B.buf.data(), B.buf.size(), cudaMemcpyHostToDevice));
     s.live = true;
-    ctx->ligs.push_back(s);
-    if (int32_t rc = sync_ligtab(ctx)) return rc;
-    *out = (ad_ligand_id)(ctx->ligs.size() - 1);
+    // the lowest free id (ids of freed ligands are reused), else a new one
+    int id = 0;
+    while (id < (int)ctx->ligs.size() && ctx->ligs[id].live) ++id;
+    if (id >= AD_MAX_LIGANDS) {
+        cudaFree(s.d_blob);
+        return fail(AD_ERR_LIMIT, "too many ligands");
+    }
+    if (id == (int)ctx->ligs.size()) ctx->ligs.push_back(s); else ctx->ligs[id] = s;
+    if (int32_t rc = sync_ligtab(ctx, id)) return rc;
+    *out = (ad_ligand_id)id;
     return AD_OK;
 }
 
 int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig) {
-    if (!ctx || lig < 0 || lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live)
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    std::lock_guard<std::mutex> lock(ctx->mu);
+    if (lig < 0 || lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live)
         return fail(AD_ERR_INVALID_ARG, "bad ligand id %d", lig);
     if (int32_t rc = set_device(ctx)) return rc;
     CUDA_TRY(cudaDeviceSynchronize());
     cudaFree(ctx->ligs[lig].d_blob);
     ctx->ligs[lig] = LigSlot{};
-    return sync_ligtab(ctx);
+    return sync_ligtab(ctx, lig);
+}
+
+int32_t ad_set_launch_ligands(ad_context* ctx, const int32_t* ids, int32_t n) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (n < 0 || (n > 0 && !ids)) return fail(AD_ERR_INVALID_ARG, "bad launch ligand list");
+    std::lock_guard<std::mutex> lock(ctx->mu);
+    for (int32_t k = 0; k < n; ++k)
+        if (ids[k] < 0 || ids[k] >= (int)ctx->ligs.size() || !ctx->ligs[ids[k]].live)
+            return fail(AD_ERR_INVALID_ARG, "launch ligand %d (entry %d) is not a live ligand", ids[k], k);
+    ctx->launch_set.assign(ids, ids + n);
+    return AD_OK;
+}
+
+int32_t ad_set_schedule_effort(ad_context* ctx, int32_t effort) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (effort < 0 || effort > 2) return fail(AD_ERR_INVALID_ARG, "schedule effort %d not in 0..2", effort);
+    std::lock_guard<std::mutex> lock(ctx->mu);
+    ctx->sched_effort = effort;
+    return AD_OK;
 }
 
 }  // extern "C"
@@ -1274,11 +1325,23 @@ WarpKernel pick_warp_kernel(int engine, bool grad, bool ls, bool wide) {
     return wide ? pick_warp_kernel_w<true>(engine, grad, ls) : pick_warp_kernel_w<false>(engine, grad, ls);
 }
 
+// The ligands a pose_ligand launch may reference: the launch set, or every live ligand.
+template <class F>
+void for_each_launch_ligand(const ad_context* ctx, F f) {
+    if (ctx->launch_set.empty()) {
+        for (const LigSlot& o : ctx->ligs)
+            if (o.live) f(o);
+    } else {
+        for (int id : ctx->launch_set)
+            if (id < (int)ctx->ligs.size() && ctx->ligs[id].live) f(ctx->ligs[id]);
+    }
+}
+
 bool launch_is_wide(const ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand) {
     if (!pose_ligand) return 6 + ctx->ligs[lig].n_tors > 32;
-    for (const LigSlot& o : ctx->ligs)
-        if (o.live && 6 + o.n_tors > 32) return true;
-    return false;
+    bool wide = false;
+    for_each_launch_ligand(ctx, [&](const LigSlot& o) { wide |= 6 + o.n_tors > 32; });
+    return wide;
 }
 
 int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const void* genes, int32_t stride) {
@@ -1294,9 +1357,10 @@ int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const 
 // pose_ligand launches may touch any live ligand; the scoring constants are kernel
 // parameters, so they must be identical across the live ligands
 int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
-    for (const LigSlot& o : ctx->ligs)
-        if (o.live && memcmp(o.ff, ctx->ligs[lig].ff, sizeof(o.ff)) != 0)
-            return fail(AD_ERR_INVALID_ARG, "pose_ligand launches need every live ligand uploaded with the same ad_ff_params");
+    bool same = true;
+    for_each_launch_ligand(ctx, [&](const LigSlot& o) { same &= memcmp(o.ff, ctx->ligs[lig].ff, sizeof(o.ff)) == 0; });
+    if (!same)
+        return fail(AD_ERR_INVALID_ARG, "pose_ligand launches need every referenced ligand uploaded with the same ad_ff_params");
     return AD_OK;
 }
 
@@ -1305,13 +1369,11 @@ int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
 int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int req_warps, cudaStream_t st,
                     bool tc_engine) {
     if (!tc_engine) L.scratch_bytes = L.scratch_simt;
-    if (p.pose_ligand) {  // any live ligand may be referenced: size for the largest footprint
-        for (const LigSlot& o : ctx->ligs)
-            if (o.live) {
-                L.blob_bytes = std::max(L.blob_bytes, o.blob_bytes);
-                L.scratch_bytes = std::max(L.scratch_bytes, tc_engine ? o.scratch_bytes : o.scratch_simt);
-            }
-    }
+    if (p.pose_ligand)  // any ligand of the launch set may be referenced: size for the largest footprint
+        for_each_launch_ligand(ctx, [&](const LigSlot& o) {
+            L.blob_bytes = std::max(L.blob_bytes, o.blob_bytes);
+            L.scratch_bytes = std::max(L.scratch_bytes, tc_engine ? o.scratch_bytes : o.scratch_simt);
+        });
     // Every pose costs the same.  A launch shape (register variant, W warps per CTA)
     // is scored by the modelled time of the busiest SM: it receives ceil(CTAs / SMs)
     // CTAs and runs them in waves of `blocks` resident CTAs; a wave of a warps
@@ -1446,11 +1508,10 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         if (6 + L.n_tors > threads) return fail(AD_ERR_INVALID_ARG, "baseline needs >= 6 + n_tors threads");
         int32_t blob = L.blob_bytes, bscr = block_scratch_layout(L.n_atoms, L.n_tors, tcec ? threads : 0).bytes;
         if (pose_ligand)
-            for (const LigSlot& o : ctx->ligs)
-                if (o.live) {
-                    blob = std::max(blob, o.blob_bytes);
-                    bscr = std::max(bscr, block_scratch_layout(o.n_atoms, o.n_tors, tcec ? threads : 0).bytes);
-                }
+            for_each_launch_ligand(ctx, [&](const LigSlot& o) {
+                blob = std::max(blob, o.blob_bytes);
+                bscr = std::max(bscr, block_scratch_layout(o.n_atoms, o.n_tors, tcec ? threads : 0).bytes);
+            });
         const size_t smem = (size_t)blob + bscr;
         if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "ligand too large for the baseline engine");
         void (*kern)(const KParams) = tcec ? k_block_baseline<true> : k_block_baseline<false>;

@@ -535,24 +535,51 @@ def make_config(cfg: int, replica: int = 0, runs: int | None = None, pop: int | 
                     iters=iters or c["iters"])
 
 
+class ScreenSpec:
+    """Config 5 as a lazy recipe: the receptor grid and the per-ligand size draws
+    up front; ligand k and its start genotypes generated on demand (a rank of a
+    sharded screen builds only its own ligands).  Seeds as in make_screen."""
+
+    def __init__(self, n_ligands: int = 8192, runs: int = 20, pop: int = 16, iters: int = 300,
+                 replica: int = 0, stride: int = 40):
+        self.seed = 5000 + replica
+        self.n_ligands, self.runs, self.pop, self.iters, self.stride = n_ligands, runs, pop, iters, stride
+        rng = np.random.default_rng(self.seed)
+        self.sizes = []
+        for _ in range(n_ligands):
+            n = int(rng.integers(20, 111))
+            t = int(rng.integers(0, min(32, n // 3) + 1))
+            self.sizes.append((n, t))
+        self.grid = make_grid(self.seed + 100, 60, TYPESETS[8], 2000)
+        self.name = "config5-screen"
+
+    def ligand(self, k: int) -> Ligand:
+        n, t = self.sizes[k]
+        return make_ligand(self.seed * 100003 + k, n, t, 8, chainlike=(n > 80))
+
+    def genes(self, k: int) -> np.ndarray:
+        """Start genotypes [runs * pop, stride] of ligand k (run-major)."""
+        return make_genotypes(self.seed + 7 * k + 1, self.runs * self.pop, self.sizes[k][1], self.grid,
+                              stride=self.stride)
+
+    def n_pairs(self, k: int) -> float:
+        """Intra-pair count ESTIMATE from the size draw (for sharding before the
+        ligands exist; only relative costs matter): pairs between the T + 1 rigid
+        fragments, ~ 0.4 n^2 (1 - 1 / (T + 1))."""
+        n, t = self.sizes[k]
+        return 0.4 * n * n * (1.0 - 1.0 / (t + 1))
+
+
 def make_screen(n_ligands: int = 8192, runs: int = 20, pop: int = 16, iters: int = 300,
                 replica: int = 0, stride: int = 40) -> Workload:
-    """Config 5: heterogeneous screen over the config-2 receptor with 8 types."""
-    seed = 5000 + replica
-    rng = np.random.default_rng(seed)
-    grid = make_grid(seed + 100, 60, TYPESETS[8], 2000)
-    ligs = []
-    for k in range(n_ligands):
-        n = int(rng.integers(20, 111))
-        t = int(rng.integers(0, min(32, n // 3) + 1))
-        ligs.append(make_ligand(seed * 100003 + k, n, t, 8, chainlike=(n > 80)))
-    n_poses = n_ligands * runs * pop
-    genes = np.zeros((n_poses, stride), dtype=np.float32)
+    """Config 5: heterogeneous screen over the config-2 receptor with 8 types
+    (every ligand and genotype materialised; ScreenSpec is the lazy form)."""
+    spec = ScreenSpec(n_ligands, runs, pop, iters, replica, stride)
+    ligs = [spec.ligand(k) for k in range(n_ligands)]
+    genes = np.concatenate([spec.genes(k) for k in range(n_ligands)]) if n_ligands else \
+        np.zeros((0, stride), dtype=np.float32)
     pl = np.repeat(np.arange(n_ligands, dtype=np.int32), runs * pop)
-    for k, lg in enumerate(ligs):
-        s = k * runs * pop
-        genes[s:s + runs * pop] = make_genotypes(seed + 7 * k + 1, runs * pop, lg.n_tors, grid, stride=stride)
-    return Workload(name="config5-screen", grid=grid, ligands=ligs, genes=genes,
+    return Workload(name=spec.name, grid=spec.grid, ligands=ligs, genes=genes,
                     pose_ligand=pl, runs=runs, pop=pop, iters=iters)
 
 

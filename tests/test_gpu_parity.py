@@ -285,6 +285,70 @@ def test_multi_ligand_pose_ligand(ctx, ad):
     _uploaded.clear()
 
 
+def test_launch_set_and_id_reuse(ad):
+    """ad_set_launch_ligands: pose_ligand launches are sized for the launch set
+    only; a pose whose ligand is outside the set's footprint is reported on the
+    next call (device-side check); freed ids are reused."""
+    grid = synth.make_grid(81, 40, synth.TYPESETS[6], 800)
+    ff = synth.FFParams()
+    c = ad.Context(0)
+    try:
+        c.upload_grid(grid)
+        small, large = synth.make_ligand(201, 16, 2, 6), synth.make_ligand(202, 60, 12, 6)
+        i_s, i_l = c.upload_ligand(small, ff), c.upload_ligand(large, ff)
+        stride = 6 + 12
+        genes = np.concatenate([synth.make_genotypes(1, 8, 2, grid, stride=stride, frac=0.3),
+                                synth.make_genotypes(2, 8, 12, grid, stride=stride, frac=0.3)])
+        pl = torch.tensor([i_s] * 8 + [i_l] * 8, dtype=torch.int32, device="cuda")
+        g = torch.from_numpy(genes).cuda()
+        E = torch.empty(16, device="cuda")
+        # the small ligand alone: the large ligand's poses must be flagged
+        c.set_launch_ligands([i_s])
+        ad.ad_score_poses(c.h, i_s, pl, g, E)
+        torch.cuda.synchronize()
+        with pytest.raises(ad.AdError):
+            ad.ad_score_poses(c.h, i_s, pl[:8], g[:8], E[:8])
+        # both ligands: every pose scores, and matches the oracle
+        c.set_launch_ligands([i_s, i_l])
+        ad.ad_score_poses(c.h, i_l, pl, g, E)
+        torch.cuda.synchronize()
+        Eh = E.cpu().numpy()
+        check_scores(small, grid, ff, genes[:8, :8], Eh[:8], label="small")
+        check_scores(large, grid, ff, genes[8:], Eh[8:], label="large")
+        with pytest.raises(ad.AdError):
+            c.set_launch_ligands([i_l + 5])  # not a live ligand
+        c.set_launch_ligands(None)
+        c.free_ligand(i_s)
+        assert c.upload_ligand(small, ff) == i_s  # lowest free id is reused
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("effort", [0, 1])
+def test_schedule_effort_parity(ad, cfg2, effort):
+    """A cheaper pair-schedule placement evaluates the same pairs: oracle parity
+    holds and energies agree with the default placement to FP32 rounding."""
+    L = cfg2.ligands[0]
+    c = ad.Context(0)
+    try:
+        c.upload_grid(cfg2.grid)
+        ref = c.upload_ligand(L, cfg2.ff)
+        c.set_schedule_effort(effort)
+        lid = c.upload_ligand(L, cfg2.ff)
+        g = torch.from_numpy(cfg2.genes[:128]).cuda()
+        E0, G0, _ = c.score(ref, g)
+        E1, G1, _ = c.score(lid, g)
+        torch.cuda.synchronize()
+        check_scores(L, cfg2.grid, cfg2.ff, cfg2.genes[:128], E1.cpu().numpy(), G1.cpu().numpy(), f"effort {effort}")
+        Eo, *_ = O.score(L, cfg2.grid, cfg2.ff, cfg2.genes[:128])
+        d = np.abs(E1.cpu().numpy().astype(np.float64) - E0.cpu().numpy())
+        assert np.all(d <= 1e-5 * np.abs(Eo) + 1e-3)
+        with pytest.raises(ad.AdError):
+            c.set_schedule_effort(3)
+    finally:
+        c.close()
+
+
 @pytest.mark.parametrize("engine", ["simt", "tc", "paper"])
 def test_reduction_engines_accuracy(ctx, ad, engine):
     """Config 4: |S - S_exact| <= (ceil(log2 P) + 2) 2^-24 sum|x| (O-7)."""
