@@ -1,30 +1,37 @@
 """NEXT-2 accuracy study: FP32 SIMT vs error-corrected TF32 (TCEC) vs FP16 without
 EC (Schieffer-Peng, Lst 1 bottom P:L236-258) reductions inside the same ADADELTA
-local search (config 2 workload, synthetic).  Reports
+local search (config 2 workload, synthetic).  Measures
   (a) per-evaluation energy / gradient error vs the FP64 oracle on relaxed poses,
   (b) per-run best energies after the full LS vs the SIMT engine: median |dE|,
       fraction worse by > 1 kcal/mol (the paper's score-success threshold),
       non-finite runs,
-  (c) the config-4 reduction error of each engine vs math.fsum.
-usage: python tools/accuracy_study.py [out.json]"""
+  (c) the config-4 reduction error of each engine vs math.fsum,
+and asserts the qualitative Fig 1 vs Fig 3 finding: the
+error-corrected TF32 engine matches FP32 SIMT, the uncorrected FP16 engine does not.
+The report is written as JSON to $AD_STUDY_OUT when set (profiles/accuracy_*.json):
+    AD_STUDY_OUT=profiles/accuracy_r01.json python -m pytest tests/test_gpu_accuracy_study.py -m gpu -s
+"""
 import json
 import math
 import os
-import sys
 
 import numpy as np
-import torch
+import pytest
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-sys.path.insert(0, ROOT)
-from oracle import oracle as O  # noqa: E402  (test infrastructure: allowed in tools/studies)
-from paper_conf_sc_solis_vasquezts25_b200 import ad, synth  # noqa: E402
+torch = pytest.importorskip("torch")
+
+from oracle import oracle as O  # noqa: E402
+from paper_conf_sc_solis_vasquezts25_b200 import synth  # noqa: E402
+
+pytestmark = pytest.mark.gpu
 
 ENG = ("simt", "tc", "tc_fp16")
 
 
-def main():
-    out_path = sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/accuracy_study.json"
+def test_accuracy_study():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_solis_vasquezts25_b200 import ad
     w = synth.make_config(2)
     L = w.ligands[0]
     Gn, stride = L.n_genes, w.genes.shape[1]
@@ -80,11 +87,15 @@ def main():
         red[e] = {"median_abs_err": float(np.median(err)), "max_abs_err": float(err.max())}
     res["reduction_256x16_uniform"] = red
     ctx.close()
-    os.makedirs(os.path.dirname(out_path) or ".", exist_ok=True)
-    with open(out_path, "w") as f:
-        json.dump(res, f, indent=1)
+    out_path = os.environ.get("AD_STUDY_OUT")
+    if out_path:
+        os.makedirs(os.path.dirname(out_path) or ".", exist_ok=True)
+        with open(out_path, "w") as f:
+            json.dump(res, f, indent=1)
     print(json.dumps(res, indent=1))
-
-
-if __name__ == "__main__":
-    main()
+    # the qualitative finding: TCEC ~ SIMT, FP16 without EC clearly worse
+    assert red["tc"]["max_abs_err"] <= 4 * red["simt"]["max_abs_err"] + 1e-6
+    assert red["tc_fp16"]["median_abs_err"] > 100 * red["tc"]["median_abs_err"]
+    assert per["tc"]["median_grad_rel_err"] <= 10 * per["simt"]["median_grad_rel_err"] + 1e-7
+    assert per["tc_fp16"]["median_grad_rel_err"] > 10 * per["tc"]["median_grad_rel_err"]
+    assert runs["tc"]["frac_worse_by_1kcal"] <= 0.05

@@ -30,7 +30,7 @@ for what in "$@"; do
       timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_block_baseline -s 1 -c 1 \
         -o gpurun_out/prof_paper_$TAG python tools/prof_ls.py 2 paper 2 > gpurun_out/ncu_paper_$TAG.log 2>&1 ;;
     accuracy)
-      timeout 900 python tools/accuracy_study.py gpurun_out/accuracy_$TAG.json > gpurun_out/accuracy_$TAG.log 2>&1; tail -3 gpurun_out/accuracy_$TAG.log ;;
+      AD_STUDY_OUT=gpurun_out/accuracy_$TAG.json timeout 900 python -m pytest tests/test_gpu_accuracy_study.py -m gpu -q -s -p no:cacheprovider > gpurun_out/accuracy_$TAG.log 2>&1; tail -3 gpurun_out/accuracy_$TAG.log ;;
     reduce)
       timeout 900 python tools/bench_reduce.py gpurun_out/reduce_$TAG.json 100 > gpurun_out/reduce_$TAG.log 2>&1; tail -25 gpurun_out/reduce_$TAG.log ;;
     ab)
