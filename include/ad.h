@@ -219,6 +219,16 @@ typedef struct {
                                threads per block for PAPER_BASELINE (0 = 64) */
     float* trace;           /* optional device [n_poses][max_iters][1 + 2*geno_stride]:
                                per evaluation E, genes, gradient (Z19 shadowed parity) */
+    int64_t* phase_cycles;  /* optional device [n_poses][5] (A14 instrumentation):
+                               clock64 cycles per pose summed over the iterations, spent in
+                               (0) pose + inter, (1) intra pairs, (2) gradient assembly
+                               (per-atom gradients, torques, gene gradients from the sums),
+                               (3) reductions (energy sum + the gene-space sums proper),
+                               (4) update (best tracking, ADADELTA).  Non-NULL runs a
+                               separately compiled instrumented kernel (SIMT, TC and the
+                               paper-style engines; AD_ERR_INVALID_ARG for TC_FP16).  The
+                               paper's reduction fraction is f = (3) / total.  Ignored by
+                               ad_lga_run. */
 } ad_ls_params;
 
 /* ADADELTA local search, one pose per warp (or per block for

@@ -52,7 +52,8 @@ class LigandDesc(C.Structure):
 
 class LSParams(C.Structure):
     _fields_ = [("max_iters", C.c_int32), ("rho", C.c_float), ("eps", C.c_float), ("pop_per_run", C.c_int32),
-                ("engine", C.c_int32), ("warps_per_cta", C.c_int32), ("trace", C.c_void_p)]
+                ("engine", C.c_int32), ("warps_per_cta", C.c_int32), ("trace", C.c_void_p),
+                ("phase_cycles", C.c_void_p)]
 
 
 class LGAParams(C.Structure):
@@ -188,10 +189,11 @@ def ad_score_poses(ctx, lig, pose_ligand, genes, energy, grad=None, aux=None, st
 
 def ad_local_search(ctx, lig, pose_ligand, genes, best_energy, run_best=None, n_evals=None, *, max_iters=300,
                     rho=0.8, eps=0.01, pop_per_run=0, engine=AD_ENGINE_SIMT, warps_per_cta=0, trace=None,
-                    stream=None) -> None:
+                    phase_cycles=None, stream=None) -> None:
     import torch
     n, stride = genes.shape
-    prm = LSParams(max_iters, rho, eps, pop_per_run, engine, warps_per_cta, _dptr(trace, torch.float32))
+    prm = LSParams(max_iters, rho, eps, pop_per_run, engine, warps_per_cta, _dptr(trace, torch.float32),
+                   _dptr(phase_cycles, torch.int64))
     _check(lib().ad_local_search(ctx, lig, _dptr(pose_ligand, torch.int32), n, _dptr(genes, torch.float32), stride,
                                  _dptr(best_energy, torch.float32), _dptr(run_best, torch.float32),
                                  _dptr(n_evals, torch.int64), C.byref(prm), _stream(stream)))
@@ -205,7 +207,7 @@ def ad_lga_run(ctx, lig, n_runs, genes, energies, run_best=None, n_evals=None, n
     n, stride = genes.shape
     assert n == n_runs * pop_size
     prm = LGAParams(pop_size, max_gens, max_evals, elitism, cross_rate, mut_rate, tour_rate, ls_rate, dmov, dang,
-                    seed, LSParams(ls_iters, rho, eps, 0, engine, warps_per_cta, None))
+                    seed, LSParams(ls_iters, rho, eps, 0, engine, warps_per_cta, None, None))
     _check(lib().ad_lga_run(ctx, lig, n_runs, _dptr(genes, torch.float32), stride, _dptr(energies, torch.float32),
                             _dptr(run_best, torch.float32), _dptr(n_evals, torch.int64), _dptr(n_gens, torch.int32),
                             C.byref(prm), _stream(stream)))
@@ -296,18 +298,20 @@ class Context:
         return E, G, A
 
     def local_search(self, lig_id, genes, *, max_iters=300, rho=0.8, eps=0.01, engine="simt", pop_per_run=0,
-                     warps_per_cta=0, trace=False, pose_ligand=None, n_evals=None):
-        """In-place LS on `genes` (CUDA tensor [n, stride]); returns dict of outputs."""
+                     warps_per_cta=0, trace=False, pose_ligand=None, n_evals=None, phases=False):
+        """In-place LS on `genes` (CUDA tensor [n, stride]); returns dict of outputs
+        (phases=True: the A14 instrumented kernel, "phase_cycles" [n, 5] int64)."""
         import torch
         n, stride = genes.shape
         dev = genes.device
         bE = torch.empty(n, dtype=torch.float32, device=dev)
         rb = torch.empty(n // pop_per_run, 1 + stride, dtype=torch.float32, device=dev) if pop_per_run else None
         tr = torch.empty(n, max_iters, 1 + 2 * stride, dtype=torch.float32, device=dev) if trace else None
+        ph = torch.zeros(n, 5, dtype=torch.int64, device=dev) if phases else None
         ad_local_search(self.h, lig_id, pose_ligand, genes, bE, rb, n_evals, max_iters=max_iters, rho=rho, eps=eps,
                         pop_per_run=pop_per_run, engine=ENGINES[engine] if isinstance(engine, str) else engine,
-                        warps_per_cta=warps_per_cta, trace=tr)
-        return {"best_energy": bE, "run_best": rb, "trace": tr}
+                        warps_per_cta=warps_per_cta, trace=tr, phase_cycles=ph)
+        return {"best_energy": bE, "run_best": rb, "trace": tr, "phase_cycles": ph}
 
     def lga(self, lig_id, genes, n_runs, *, engine="simt", **kw):
         """NEXT-3 Lamarckian GA in place on `genes` (CUDA [n_runs * pop_size, stride])."""

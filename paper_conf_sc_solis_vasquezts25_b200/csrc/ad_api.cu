@@ -1311,6 +1311,17 @@ WarpKernel wk() {
     return WarpKernel{k_warp_engine<E, GR, LS, AD_WARP_MAXNREG, W>, k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W>};
 }
 
+// A14 instrumented LS kernels (ad_ls_params.phase_cycles): SIMT and TC engines
+template <int E, bool W>
+WarpKernel wk_instr() {
+    return WarpKernel{k_warp_engine<E, true, true, AD_WARP_MAXNREG, W, true>,
+                      k_warp_engine<E, true, true, AD_WARP_MAXNREG_HI, W, true>};
+}
+WarpKernel pick_instr_kernel(int engine, bool wide) {
+    if (engine == AD_ENGINE_TC) return wide ? wk_instr<1, true>() : wk_instr<1, false>();
+    return wide ? wk_instr<0, true>() : wk_instr<0, false>();
+}
+
 template <bool W>
 WarpKernel pick_warp_kernel_w(int engine, bool grad, bool ls) {
     if (ls) return engine == AD_ENGINE_TC        ? wk<1, true, true, W>()
@@ -1500,6 +1511,9 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     p.max_iters = prm->max_iters;
     p.rho = prm->rho;
     p.eps = prm->eps;
+    p.phase_cycles = prm->phase_cycles;
+    if (p.phase_cycles && prm->engine == AD_ENGINE_TC_FP16)
+        return fail(AD_ERR_INVALID_ARG, "phase_cycles: no instrumented build of the TC_FP16 engine");
     const LigSlot& L = ctx->ligs[lig];
     if (prm->engine == AD_ENGINE_PAPER_BASELINE || prm->engine == AD_ENGINE_PAPER_TCEC) {
         const bool tcec = prm->engine == AD_ENGINE_PAPER_TCEC;
@@ -1514,7 +1528,8 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
             });
         const size_t smem = (size_t)blob + bscr;
         if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "ligand too large for the baseline engine");
-        void (*kern)(const KParams) = tcec ? k_block_baseline<true> : k_block_baseline<false>;
+        void (*kern)(const KParams) = p.phase_cycles ? (tcec ? k_block_baseline<true, true> : k_block_baseline<false, true>)
+                                                     : (tcec ? k_block_baseline<true> : k_block_baseline<false>);
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         p.smem_blob = blob;
         p.smem_scratch = bscr;
@@ -1526,8 +1541,10 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     } else {
         int w = prm->warps_per_cta;
         if (w < 0 || w > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..16", w);
-        if (int32_t rc = launch_warp(ctx, L, pick_warp_kernel(prm->engine, true, true, launch_is_wide(ctx, lig, pose_ligand)), p, w, st,
-                                     prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16))
+        const bool wide = launch_is_wide(ctx, lig, pose_ligand);
+        const WarpKernel k = p.phase_cycles ? pick_instr_kernel(prm->engine, wide)
+                                            : pick_warp_kernel(prm->engine, true, true, wide);
+        if (int32_t rc = launch_warp(ctx, L, k, p, w, st, prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16))
             return rc;
     }
     if (run_best) {

@@ -217,7 +217,11 @@ struct KParams {
     int32_t smem_scratch;   // bytes per warp (SIMT/TC) or per block (baseline)
     int32_t n_ligs;
     const int32_t* n_active;  // optional device count: poses >= *n_active exit (LGA's compacted LS list)
+    int64_t* phase_cycles;    // A14 instrumented kernels only: [n_poses][PH_N] clock64 cycles per phase
 };
+
+// A14 phases (ad_ls_params.phase_cycles): indices of the per-pose cycle counters
+enum Phase { PH_POSE_INTER = 0, PH_INTRA = 1, PH_ASSEMBLE = 2, PH_REDUCE = 3, PH_UPDATE = 4, PH_N = 5 };
 
 // NEXT-3 GA generation parameters (ad_lga_params minus the LS part)
 struct GaParams {

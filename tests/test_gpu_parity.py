@@ -349,6 +349,32 @@ def test_schedule_effort_parity(ad, cfg2, effort):
         c.close()
 
 
+@pytest.mark.parametrize("engine", ["simt", "tc", "paper", "paper_tcec"])
+def test_phase_instrumentation(ctx, cfg2, engine):
+    """A14: the instrumented kernel computes exactly what the plain kernel computes
+    (same arithmetic, FMA contraction off) and reports positive cycles for every
+    phase; the reduction share f is a proper fraction."""
+    (lid,) = _setup(ctx, cfg2, "cfg2")
+    wpc = 64 if engine.startswith("paper") else 0
+    outs = []
+    for phases in (False, True):
+        g = torch.from_numpy(cfg2.genes[:300]).cuda()
+        o = ctx.local_search(lid, g, max_iters=20, engine=engine, warps_per_cta=wpc, phases=phases)
+        torch.cuda.synchronize()
+        outs.append((o["best_energy"].cpu().numpy(), g.cpu().numpy(), o["phase_cycles"]))
+    if engine.startswith("paper"):
+        # the paper-style kernel accumulates intra gradients with shared-memory float
+        # atomics (order not fixed): equal up to rounding, not bit for bit
+        d = np.abs(outs[0][0].astype(np.float64) - outs[1][0])
+        assert np.mean(d > 1e-2 * (1 + np.abs(outs[0][0]))) < 0.05
+    else:
+        assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    ph = outs[1][2].cpu().numpy()
+    assert ph.shape == (300, 5) and np.all(ph > 0)
+    f = ph[:, 3].sum() / ph.sum()
+    assert 0.0 < f < 0.5
+
+
 @pytest.mark.parametrize("engine", ["simt", "tc", "paper"])
 def test_reduction_engines_accuracy(ctx, ad, engine):
     """Config 4: |S - S_exact| <= (ceil(log2 P) + 2) 2^-24 sum|x| (O-7)."""
