@@ -113,7 +113,7 @@ struct GridDev {
 struct WarpScratch {
     int32_t x;      // float4 [Npad]        world coords + charge
     int32_t g;      // float4 [K][Npad]+8   atom gradient accumulators (slot 0 seeded with inter) + 8 spare
-    int32_t w;      // float4 [Npad+1][2]   prefix sums (SIMT) / W staging (TC)
+    int32_t w;      // float4 [Npad+1][2]   W staging (TC engines only)
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
     int32_t trig;   // float2 [T]           cos, sin of torsion angles
     int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
@@ -135,12 +135,16 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     // rows of npad float4 (slot k of atom a at k * npad + a) + the start of a spare
     // row K: empty schedule places only ever target K * npad + (0..7)
     s.g = o;     o += 16 * npad * n_slots + 16 * 8;
-    s.w = o;     o += 32 * (npad + 1);
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
     s.genes = o; o += 4 * kMaxGenes;
     s.part = o;  o += 16 * 32 * n_chunks;
-    s.bytes_simt = o;                               // the SIMT engine needs no D tile
+    // the SIMT engine needs neither W nor D: its prefix sums overwrite the X and
+    // slot-0 gradient rows the scan has just consumed (ad_kernels.cuh, a4-a5), so
+    // its per-warp footprint ends here (a smaller shared-memory carve-out leaves
+    // more L1 for the grid gathers)
+    s.bytes_simt = o;
+    s.w = o;     o += 32 * (npad + 1);              // TC engines: W staging
     s.d = o;     o += align16(4 * 8 * mpad);
     s.bytes = o;
     return s;
