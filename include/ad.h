@@ -215,7 +215,7 @@ typedef struct {
     float rho, eps;         /* decay and conditioning constants (0.8, 0.01; Z14) */
     int32_t pop_per_run;    /* poses per run for run_best; 0 = no run_best */
     int32_t engine;         /* enum ad_engine */
-    int32_t warps_per_cta;  /* poses per CTA for SIMT/TC/TC_FP16, 0..16 (0 = library choice);
+    int32_t warps_per_cta;  /* poses per CTA for SIMT/TC/TC_FP16, 0..32 (0 = library choice);
                                threads per block for PAPER_BASELINE (0 = 64) */
     float* trace;           /* optional device [n_poses][max_iters][1 + 2*geno_stride]:
                                per evaluation E, genes, gradient (Z19 shadowed parity) */

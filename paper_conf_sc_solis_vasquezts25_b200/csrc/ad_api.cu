@@ -1395,17 +1395,18 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // (22 poses) 3.87, W = 8 (24 poses) 4.02.  The 128-register twin executes
     // ~10 % fewer instructions and no spills: its time is scaled by 0.85 (config 3,
     // smem-bound at 16 warps/SM either way: 128.3 ms vs 147.7 ms for the 80-register
-    // twin at 18).  Ties: more resident warps, then fewer CTAs (fewer blob stagings).
+    // twin at 18).  Ties: less shared memory in use per SM (fewer blob copies: more L1
+    // left for the grid gathers and spills), then more resident warps.
     // Mixed-ligand launches keep power-of-two CTA sizes (pose_ligand groups stay aligned).
-    struct Cand { int w = 0, active = -1; double cost = 1e300; long ctas = 0; size_t smem = 0; WarpKernelFn k = nullptr; };
+    struct Cand { int w = 0, active = -1; double cost = 1e300; size_t sm_smem = 0; size_t smem = 0; WarpKernelFn k = nullptr; };
     Cand pick;
     static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
     for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
         if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
-        for (int w = 1; w <= 16; ++w) {
+        for (int w = 1; w <= 32; ++w) {
             if (req_warps > 0 && w != req_warps) continue;
-            if (p.pose_ligand && (w & (w - 1))) continue;
+            if (p.pose_ligand && ((w & (w - 1)) || w > 8)) continue;  // ad.h: ligand runs are multiples of 8
             const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
             if (smem > (size_t)ctx->max_smem_optin) continue;
             CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -1422,9 +1423,10 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             if (getenv("AD_DEBUG_LAUNCH"))
                 fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld per_sm=%ld cost=%.3f\n",
                         v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, per_sm, cost);
+            const size_t sm_smem = (size_t)std::min<long>(blocks, per_sm) * smem;  // in use on the busiest SM
             const bool better = cost < pick.cost - 1e-9 ||
-                                (cost < pick.cost + 1e-9 && (active > pick.active || (active == pick.active && ctas < pick.ctas)));
-            if (better) pick = Cand{w, active, cost, ctas, smem, k};
+                                (cost < pick.cost + 1e-9 && (sm_smem < pick.sm_smem || (sm_smem == pick.sm_smem && active > pick.active)));
+            if (better) pick = Cand{w, active, cost, sm_smem, smem, k};
         }
     }
     const int best_w = pick.w, best_active = pick.active;
@@ -1540,7 +1542,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         CUDA_TRY(cudaGetLastError());
     } else {
         int w = prm->warps_per_cta;
-        if (w < 0 || w > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..16", w);
+        if (w < 0 || w > 32) return fail(AD_ERR_INVALID_ARG, "warps_per_cta %d not in 0..32", w);
         const bool wide = launch_is_wide(ctx, lig, pose_ligand);
         const WarpKernel k = p.phase_cycles ? pick_instr_kernel(prm->engine, wide)
                                             : pick_warp_kernel(prm->engine, true, true, wide);
@@ -1575,7 +1577,7 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
         return fail(AD_ERR_INVALID_ARG, "LGA runs the warp engines (SIMT, TC, TC_FP16)");
     if (ls.max_iters < 1 || !(ls.rho >= 0.f && ls.rho < 1.f) || !(ls.eps > 0.f))
         return fail(AD_ERR_INVALID_ARG, "bad LS parameters");
-    if (ls.warps_per_cta < 0 || ls.warps_per_cta > 16) return fail(AD_ERR_INVALID_ARG, "warps_per_cta not in 0..16");
+    if (ls.warps_per_cta < 0 || ls.warps_per_cta > 32) return fail(AD_ERR_INVALID_ARG, "warps_per_cta not in 0..32");
     if (prm->elitism < 0 || prm->elitism > pop || prm->max_gens < 0 || prm->max_evals < 0)
         return fail(AD_ERR_INVALID_ARG, "bad GA parameters");
     if (int32_t rc = set_device(ctx)) return rc;
