@@ -55,7 +55,8 @@ int32_t fail(int32_t code, const char* fmt, ...) {
 
 struct LigSlot {
     unsigned char* d_blob = nullptr;
-    int32_t blob_bytes = 0;
+    int32_t blob_bytes = 0;      // staged by the warp engine
+    int32_t base_bytes = 0;      // staged by the paper-style baseline
     int32_t scratch_bytes = 0;   // per warp (TC engine)
     int32_t scratch_simt = 0;    // per warp (SIMT engine)
     int32_t block_scratch = 0;   // per block (baseline)
@@ -86,6 +87,7 @@ struct ad_context {
     int32_t last_grid = 0, last_block = 0, last_smem = 0, last_maxreg = 0;
     // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
     int32_t pairs_smem_max = 16384;
+    int32_t pk_smem_max = 32768;  // packed schedule bytes (32 per place) staged per CTA at most
     // host effort spent on the pair schedule's bank-conflict placement (ad_set_schedule_effort)
     int32_t sched_effort = 2;
     // ligands that pose_ligand launches may reference (ad_set_launch_ligands; empty = every
@@ -123,7 +125,7 @@ int32_t sync_ligtab(ad_context* ctx, int only = -1) {
     const int n = (int)ctx->ligs.size();
     if (only >= 0 && only < ctx->ligtab_cap) {
         const LigSlot& L = ctx->ligs[only];
-        const LigDev e{L.live ? L.d_blob : nullptr, L.blob_bytes, L.scratch_bytes, L.scratch_simt, 0};
+        const LigDev e{L.live ? L.d_blob : nullptr, L.blob_bytes, L.scratch_bytes, L.scratch_simt, L.base_bytes};
         CUDA_TRY(cudaMemcpy(ctx->d_ligtab + only, &e, sizeof(LigDev), cudaMemcpyHostToDevice));
         return AD_OK;
     }
@@ -139,7 +141,7 @@ int32_t sync_ligtab(ad_context* ctx, int only = -1) {
     std::vector<LigDev> h(n);
     for (int i = 0; i < n; ++i)
         h[i] = LigDev{ctx->ligs[i].live ? ctx->ligs[i].d_blob : nullptr, ctx->ligs[i].blob_bytes,
-                      ctx->ligs[i].scratch_bytes, ctx->ligs[i].scratch_simt, 0};
+                      ctx->ligs[i].scratch_bytes, ctx->ligs[i].scratch_simt, ctx->ligs[i].base_bytes};
     if (n) CUDA_TRY(cudaMemcpy(ctx->d_ligtab, h.data(), sizeof(LigDev) * n, cudaMemcpyHostToDevice));
     return AD_OK;
 }
@@ -883,6 +885,7 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
     if (!ctx) return fail(AD_ERR_OOM, "host allocation failed");
     ctx->device = cuda_device;
     if (const char* m = getenv("AD_PAIRS_SMEM_MAX")) ctx->pairs_smem_max = atoi(m);
+    if (const char* m = getenv("AD_PK_SMEM_MAX")) ctx->pk_smem_max = atoi(m);  // 0: no packed schedules (A/B)
     if (const char* m = getenv("AD_INTRA_MODE"))
         ctx->intra_mode = strcmp(m, "owner") == 0 ? INTRA_OWNER : strcmp(m, "hybrid") == 0 ? INTRA_HYBRID : INTRA_SCATTER;
     cudaError_t e = cudaSetDevice(cuda_device);
@@ -1221,9 +1224,43 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     // through L1, one copy per SM) instead of being staged into every CTA
     H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
     H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
-    H.blob_bytes = (int32_t)B.buf.size();
-    const int32_t pair_bytes = H.blob_bytes - H.off_prec;
+    const int32_t pair_bytes = (int32_t)B.buf.size() - H.off_prec;
     H.pairs_gmem = pair_bytes > ctx->pairs_smem_max ? 1 : 0;
+    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
+    // packed schedule (see ad_internal.h): scatter mode, schedule in shared memory,
+    // every row byte offset below 64 KiB
+    const int n_places = sch.rounds * kPairsPerStep;
+    const bool packed = mode == INTRA_SCATTER && !H.pairs_gmem && n_places > 0 &&
+                        n_places * 32 <= ctx->pk_smem_max && ws.g + 16 * (H.n_pad * (sch.slots + 1)) <= 0xffff;
+    H.off_pk = 0;
+    const int32_t base_bytes = (int32_t)B.buf.size();
+    if (packed) {
+        std::vector<uint4> pka(n_places);
+        std::vector<float4> pkb(n_places);
+        const float delta = H.ff[FF_DELTA];
+        for (int q = 0; q < n_places; ++q) {
+            const uint32_t rec = sch.rec[q];
+            const uint32_t i = rec & 0xffu, si = (rec >> 16) & 0xfu, sj = (rec >> 20) & 0xfu;
+            uint32_t j = (rec >> 8) & 0xffu;
+            const bool empty = (int)si == sch.slots;
+            // an empty place reads two X rows; with no smoothing band (delta = 0) they
+            // must differ, or its zero coefficients would multiply 1/0
+            if (empty && j == i && delta == 0.f) j = (i + 1) % (uint32_t)N;
+            const uint32_t gi = (uint32_t)ws.g + 16u * (si * (uint32_t)H.n_pad + i);
+            const uint32_t gj = (uint32_t)ws.g + 16u * (sj * (uint32_t)H.n_pad + ((rec >> 8) & 0xffu));
+            float dsv = sch.dsv[2 * q], cqq = sch.dsv[2 * q + 1];
+            float4 c = tp[rec >> 24];
+            if (empty) { c.x = 0.f; c.y = 0.f; dsv = 0.f; cqq = 0.f; }
+            uint32_t ub, uc;
+            memcpy(&ub, &dsv, 4);
+            memcpy(&uc, &cqq, 4);
+            pka[q] = make_uint4((16u * i) | ((16u * j) << 16), gi | (gj << 16), ub, uc);
+            pkb[q] = c;
+        }
+        H.off_pk = B.put(pka.data(), sizeof(uint4) * pka.size());
+        B.put(pkb.data(), sizeof(float4) * pkb.size());
+    }
+    H.blob_bytes = (int32_t)B.buf.size();
     if (const char* dump = getenv("AD_DUMP_SCHEDULE")) {  // debugging aid: raw schedule records
         if (FILE* f = fopen(dump, "ab")) {
             const int32_t hdr[4] = {N, sch.rounds, sch.slots, H.n_pad};
@@ -1233,7 +1270,6 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         }
     }
     H.stage_bytes = H.pairs_gmem ? H.off_prec : H.blob_bytes;
-    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
     H.scratch_bytes = ws.bytes;
     H.ws_g = ws.g; H.ws_w = ws.w; H.ws_d = ws.d; H.ws_trig = ws.trig;
     H.ws_tw = ws.tw; H.ws_genes = ws.genes; H.ws_part = ws.part;
@@ -1242,7 +1278,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     std::lock_guard<std::mutex> lock(ctx->mu);
     if (int32_t rc = set_device(ctx)) return rc;
     LigSlot s;
-    s.blob_bytes = H.stage_bytes;  // shared-memory bytes staged per CTA
+    s.blob_bytes = H.stage_bytes;  // shared-memory bytes staged per CTA (warp engine)
+    s.base_bytes = H.pairs_gmem ? H.off_prec : base_bytes;  // paper-style baseline: no packed schedule
     s.scratch_bytes = ws.bytes;
     s.scratch_simt = ws.bytes_simt;
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
@@ -1522,10 +1559,10 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         int threads = prm->warps_per_cta > 0 ? prm->warps_per_cta : 64;
         if (threads % 32 || threads < 32 || threads > 256) return fail(AD_ERR_INVALID_ARG, "baseline block size %d", threads);
         if (6 + L.n_tors > threads) return fail(AD_ERR_INVALID_ARG, "baseline needs >= 6 + n_tors threads");
-        int32_t blob = L.blob_bytes, bscr = block_scratch_layout(L.n_atoms, L.n_tors, tcec ? threads : 0).bytes;
+        int32_t blob = L.base_bytes, bscr = block_scratch_layout(L.n_atoms, L.n_tors, tcec ? threads : 0).bytes;
         if (pose_ligand)
             for_each_launch_ligand(ctx, [&](const LigSlot& o) {
-                blob = std::max(blob, o.blob_bytes);
+                blob = std::max(blob, o.base_bytes);
                 bscr = std::max(bscr, block_scratch_layout(o.n_atoms, o.n_tors, tcec ? threads : 0).bytes);
             });
         const size_t smem = (size_t)blob + bscr;

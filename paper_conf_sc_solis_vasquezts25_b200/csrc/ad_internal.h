@@ -24,6 +24,15 @@
 //            partial slots k*32+lane that belong to atom a)
 //   tp      float4 [nt*nt*8] cA, cB, r0, n (m == 12); 8 copies per entry (index t*8+c),
 //                           lane l reads copy l%8 -> conflict-free 128-bit lookups
+//   pka     u32x4  [R*64]   (packed schedule, off_pk != 0: INTRA_SCATTER with the schedule
+//                           in shared memory) the same places as prec, pre-decoded:
+//                           {X row byte offsets i | j<<16, gradient row byte offsets
+//                           (per-warp scratch relative, slot * npad + row) i | j<<16,
+//                           dsv bits, cqq bits}
+//   pkb     float4 [R*64]   cA, cB, r0, n of the place; empty places: cA = cB = dsv = cqq
+//                           = 0 (their E and dE/dr are exactly 0; no per-place select)
+//           The warp engine stages the whole blob; the paper-style baseline stages
+//           [0, off_pk) (prec / pdsv / tp), its footprint unchanged.
 //
 // Per-warp scratch (after the blob, one slice per warp), see WarpScratch below.
 #pragma once
@@ -77,7 +86,8 @@ struct alignas(16) LigHeader {
     int32_t n_entries, n_chunks, off_comb, off_combidx; // 96  (owner mode: E per lane, chunks per lane)
     int32_t pairs_gmem, stage_bytes, ws_g, ws_w;        // 112: schedule in global memory?, bytes staged to smem
     int32_t ws_d, ws_trig, ws_tw, ws_genes;             // 128  per-warp scratch offsets (WarpScratch, ws_x = 0),
-    int32_t ws_part, reserved0, reserved1, reserved2;   // 144  precomputed so kernels reload, not recompute, them
+    int32_t ws_part, off_pk, reserved1, reserved2;      // 144  precomputed so kernels reload, not recompute, them;
+                                                        //      off_pk: packed schedule (0 = none)
     float ff[FF_N];                                     // 208
 };
 static_assert(sizeof(LigHeader) == 208, "header size");
@@ -85,10 +95,10 @@ static_assert(sizeof(LigHeader) == 208, "header size");
 // Device table entry, one per uploaded ligand.
 struct LigDev {
     const unsigned char* blob;  // global copy of the whole blob
-    int32_t blob_bytes;         // bytes staged into shared memory (header .. tables [.. schedule])
+    int32_t blob_bytes;         // bytes the warp engine stages into shared memory (header .. tables [.. schedule])
     int32_t scratch_bytes;      // per-warp scratch, TC engine
     int32_t scratch_simt;       // per-warp scratch, SIMT engine (no D tile)
-    int32_t pad;
+    int32_t base_bytes;         // bytes the paper-style baseline stages (no packed schedule)
 };
 
 // Grid in device memory, x-pair layout:
