@@ -87,7 +87,7 @@ struct ad_context {
     int32_t last_grid = 0, last_block = 0, last_smem = 0, last_maxreg = 0;
     // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
     int32_t pairs_smem_max = 16384;
-    int32_t pk_smem_max = 32768;  // packed schedule bytes (32 per place) staged per CTA at most
+    int32_t pk_smem_max = 32768;  // packed schedule bytes (24 per place) staged per CTA at most
     // host effort spent on the pair schedule's bank-conflict placement (ad_set_schedule_effort)
     int32_t sched_effort = 2;
     // ligands that pose_ligand launches may reference (ad_set_launch_ligands; empty = every
@@ -1231,34 +1231,32 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     // every row byte offset below 64 KiB
     const int n_places = sch.rounds * kPairsPerStep;
     const bool packed = mode == INTRA_SCATTER && !H.pairs_gmem && n_places > 0 &&
-                        n_places * 32 <= ctx->pk_smem_max && ws.g + 16 * (H.n_pad * (sch.slots + 1)) <= 0xffff;
+                        n_places * 24 <= ctx->pk_smem_max && ws.g + 16 * (H.n_pad * (sch.slots + 1)) <= 0xffff;
     H.off_pk = 0;
     const int32_t base_bytes = (int32_t)B.buf.size();
     if (packed) {
         std::vector<uint4> pka(n_places);
-        std::vector<float4> pkb(n_places);
-        const float delta = H.ff[FF_DELTA];
+        std::vector<float2> pkb(n_places);
+        const uint32_t npad = (uint32_t)H.n_pad;
         for (int q = 0; q < n_places; ++q) {
             const uint32_t rec = sch.rec[q];
-            const uint32_t i = rec & 0xffu, si = (rec >> 16) & 0xfu, sj = (rec >> 20) & 0xfu;
-            uint32_t j = (rec >> 8) & 0xffu;
-            const bool empty = (int)si == sch.slots;
-            // an empty place reads two X rows; with no smoothing band (delta = 0) they
-            // must differ, or its zero coefficients would multiply 1/0
-            if (empty && j == i && delta == 0.f) j = (i + 1) % (uint32_t)N;
-            const uint32_t gi = (uint32_t)ws.g + 16u * (si * (uint32_t)H.n_pad + i);
-            const uint32_t gj = (uint32_t)ws.g + 16u * (sj * (uint32_t)H.n_pad + ((rec >> 8) & 0xffu));
-            float dsv = sch.dsv[2 * q], cqq = sch.dsv[2 * q + 1];
-            float4 c = tp[rec >> 24];
-            if (empty) { c.x = 0.f; c.y = 0.f; dsv = 0.f; cqq = 0.f; }
-            uint32_t ub, uc;
-            memcpy(&ub, &dsv, 4);
-            memcpy(&uc, &cqq, 4);
-            pka[q] = make_uint4((16u * i) | ((16u * j) << 16), gi | (gj << 16), ub, uc);
-            pkb[q] = c;
+            const uint32_t i = rec & 0xffu, j = (rec >> 8) & 0xffu, si = (rec >> 16) & 0xfu, sj = (rec >> 20) & 0xfu;
+            const uint32_t gi = (uint32_t)ws.g + 16u * (si * npad + i);
+            const uint32_t gj = (uint32_t)ws.g + 16u * (sj * npad + j);
+            if ((int)si == sch.slots) {  // empty place: the zero-charge rows, zero coefficients, spare row
+                pka[q] = make_uint4((16u * npad) | ((16u * (npad + 1)) << 16), gi | (gj << 16), 0u, 0u);
+                pkb[q] = make_float2(0.f, 1.f);
+                continue;
+            }
+            const float4 c = tp[rec >> 24];
+            uint32_t ud, ua;
+            memcpy(&ud, &sch.dsv[2 * q], 4);
+            memcpy(&ua, &c.x, 4);
+            pka[q] = make_uint4((16u * i) | ((16u * j) << 16), gi | (gj << 16), ud, ua);
+            pkb[q] = make_float2(c.y, c.w > 8.f ? -c.z : c.z);  // sign bit = 12-10 (H-bond) pair
         }
         H.off_pk = B.put(pka.data(), sizeof(uint4) * pka.size());
-        B.put(pkb.data(), sizeof(float4) * pkb.size());
+        B.put(pkb.data(), sizeof(float2) * pkb.size());
     }
     H.blob_bytes = (int32_t)B.buf.size();
     if (const char* dump = getenv("AD_DUMP_SCHEDULE")) {  // debugging aid: raw schedule records

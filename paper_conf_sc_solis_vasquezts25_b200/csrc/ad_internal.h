@@ -28,9 +28,11 @@
 //                           in shared memory) the same places as prec, pre-decoded:
 //                           {X row byte offsets i | j<<16, gradient row byte offsets
 //                           (per-warp scratch relative, slot * npad + row) i | j<<16,
-//                           dsv bits, cqq bits}
-//   pkb     float4 [R*64]   cA, cB, r0, n of the place; empty places: cA = cB = dsv = cqq
-//                           = 0 (their E and dE/dr are exactly 0; no per-place select)
+//                           dsv bits, cA bits}
+//   pkb     float2 [R*64]   cB, r0 with the sign bit set for n = 10 (H-bond).  The
+//                           kernel forms coeff_el q_i q_j from the X rows' charges.
+//                           Empty places read the two zero-charge X rows with
+//                           cA = cB = dsv = 0: their E and dE/dr are exactly 0.
 //           The warp engine stages the whole blob; the paper-style baseline stages
 //           [0, off_pk) (prec / pdsv / tp), its footprint unchanged.
 //
@@ -121,7 +123,7 @@ struct GridDev {
 
 // Per-warp scratch layout (offsets in bytes from the warp's slice; 16-aligned).
 struct WarpScratch {
-    int32_t x;      // float4 [Npad]        world coords + charge
+    int32_t x;      // float4 [Npad+2]      world coords + charge (+ 2 zero-charge rows)
     int32_t g;      // float4 [K][Npad]+8   atom gradient accumulators (slot 0 seeded with inter) + 8 spare
     int32_t w;      // float4 [Npad+1][2]   W staging (TC engines only)
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
@@ -141,7 +143,9 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     const int32_t npad = (n_atoms + 7) & ~7;
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
     int32_t o = 0;
-    s.x = o;     o += 16 * npad;
+    // X rows + two zero-charge rows (positions (0,0,0), (1,0,0)) that the empty
+    // places of packed schedules read
+    s.x = o;     o += 16 * (npad + 2);
     // rows of npad float4 (slot k of atom a at k * npad + a) + the start of a spare
     // row K: empty schedule places only ever target K * npad + (0..7)
     s.g = o;     o += 16 * npad * n_slots + 16 * 8;
