@@ -87,7 +87,7 @@ struct ad_context {
     int32_t last_grid = 0, last_block = 0, last_smem = 0, last_maxreg = 0;
     // pair schedules above this size are read from global memory (AD_PAIRS_SMEM_MAX)
     int32_t pairs_smem_max = 16384;
-    int32_t pk_smem_max = 32768;  // packed schedule bytes (24 per place) staged per CTA at most
+    int32_t pk_smem_max = 32768;  // cherry-schedule record bytes (48 per lane-step) staged per CTA at most
     // host effort spent on the pair schedule's bank-conflict placement (ad_set_schedule_effort)
     int32_t sched_effort = 2;
     // ligands that pose_ligand launches may reference (ad_set_launch_ligands; empty = every
@@ -684,6 +684,353 @@ Schedule schedule_pairs(int n_atoms, const std::vector<int>& pi, const std::vect
     return best;
 }
 
+// ---------------------------------------------------------------------------
+// Cherry schedule: the shared-memory mode of INTRA_SCATTER (kernel side:
+// intra_cherry).  Rows are storage rows (< npad).
+//   (1) cherries: every pair becomes an end of a cherry (c; e0, e1) = the pairs
+//       (c, e0), (c, e1).  Atoms are visited by descending degree; each pairs up
+//       its remaining pairs two by two as cherries centred on itself, holding one
+//       back (towards an unvisited atom) when the count is odd.  A connected pair
+//       graph with an even pair count decomposes completely into cherries; what is
+//       left over becomes a single (one empty end).  High-degree atoms become
+//       centres, which evens out the per-atom target load (a centre is ONE
+//       gradient target for two pairs).
+//   (2) steps: greedy first-fit of the cherries into steps of 32 lanes with at
+//       most K targets per atom and step (slots 0..K-1): the smallest K reaching
+//       the fewest steps.  Capped at 4 centres and 8 ends per bank group and step
+//       (a precondition of a conflict-free placement) unless the cap costs a step.
+//   (3) placement: local search over the lane positions (quarter-warps of 8
+//       lanes; swaps within and across steps that keep every step within K
+//       targets per atom) and the end order of every cherry, minimising the
+//       shared-memory wavefronts: sum over quarter-warps and the three 128-bit
+//       accesses (centre, end 0, end 1) of the largest number of lanes sharing a
+//       bank group (row % 8; X rows and gradient rows of an atom share it, npad %
+//       8 == 0).  Config 2 reaches 13.5 wavefronts per step-quarter set (ideal 12).
+struct CherryLane {
+    int c = -1, e[2] = {-1, -1}, p[2] = {-1, -1};  // rows; pair ids (-1: empty end / lane)
+    int kc = -1, ke[2] = {-1, -1};                  // slots of the targets
+};
+struct CherrySchedule {
+    int steps = 0, slots = 1;
+    std::vector<CherryLane> lane;  // [steps * 32]
+};
+
+std::vector<CherryLane> make_cherries(int n_idx, const std::vector<int>& pi, const std::vector<int>& pj) {
+    const int P = (int)pi.size();
+    std::vector<std::vector<int>> inc(n_idx);
+    for (int q = 0; q < P; ++q) {
+        inc[pi[q]].push_back(q);
+        inc[pj[q]].push_back(q);
+    }
+    std::vector<int> order(n_idx);
+    for (int a = 0; a < n_idx; ++a) order[a] = a;
+    std::stable_sort(order.begin(), order.end(), [&](int x, int y) { return inc[x].size() > inc[y].size(); });
+    std::vector<char> used(P, 0), visited(n_idx, 0);
+    auto other = [&](int q, int a) { return pi[q] == a ? pj[q] : pi[q]; };
+    std::vector<CherryLane> out;
+    for (int a : order) {
+        std::vector<int> rem;
+        for (int q : inc[a])
+            if (!used[q]) rem.push_back(q);
+        visited[a] = 1;
+        if (rem.size() % 2)  // hold back one pair towards an unvisited atom: it pairs up there
+            for (size_t k = 0; k < rem.size(); ++k)
+                if (!visited[other(rem[k], a)]) {
+                    rem.erase(rem.begin() + (long)k);
+                    break;
+                }
+        // two pairs of one cherry must end on different atoms (duplicate pairs)
+        while (rem.size() >= 2) {
+            const int q0 = rem.back();
+            rem.pop_back();
+            size_t k = rem.size();
+            while (k > 0 && other(rem[k - 1], a) == other(q0, a)) --k;
+            if (k == 0) break;  // q0 stays unused: a single below
+            const int q1 = rem[k - 1];
+            rem.erase(rem.begin() + (long)(k - 1));
+            CherryLane L;
+            L.c = a;
+            L.e[0] = other(q0, a);
+            L.e[1] = other(q1, a);
+            L.p[0] = q0;
+            L.p[1] = q1;
+            used[q0] = used[q1] = 1;
+            out.push_back(L);
+        }
+    }
+    for (int q = 0; q < P; ++q)
+        if (!used[q]) {
+            CherryLane L;
+            L.c = pi[q];
+            L.e[0] = pj[q];
+            L.p[0] = q;
+            out.push_back(L);
+        }
+    return out;
+}
+
+// wavefronts of one quarter-warp (8 lanes): sum over the three accesses of the
+// largest number of lanes in one bank group; empty ends / lanes do not count
+// (they get a free bank group later)
+int cherry_quarter_cost(const CherryLane* const* q, const uint8_t* flip) {
+    int cost = 0;
+    for (int acc = 0; acc < 3; ++acc) {
+        int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0}, mx = 0;
+        for (int l = 0; l < 8; ++l) {
+            if (!q[l] || q[l]->c < 0) continue;
+            const int row = acc == 0 ? q[l]->c : q[l]->e[(acc - 1) ^ flip[l]];
+            if (row < 0) continue;
+            mx = std::max(mx, ++cnt[row & 7]);
+        }
+        cost += mx;
+    }
+    return cost;
+}
+
+// max_steps: a schedule with more steps is not placed (steps is still reported)
+CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const std::vector<int>& pj, int effort,
+                                 int max_steps = 1 << 30) {
+    CherrySchedule S;
+    std::vector<CherryLane> ch = make_cherries(n_idx, pi, pj);
+    const int n = (int)ch.size();
+    if (n == 0) return S;
+    {  // deterministic shuffle (first-fit order)
+        uint64_t st = 0x2545F4914F6CDD1Dull;
+        for (int q = n - 1; q > 0; --q) {
+            st ^= st << 13; st ^= st >> 7; st ^= st << 17;
+            std::swap(ch[q], ch[(int)(st % (uint64_t)(q + 1))]);
+        }
+    }
+    const int target = (n + 31) / 32;
+    std::vector<std::vector<int>> best;
+    int bestK = 0;
+    for (int capped = 1; capped >= 0; --capped) {
+        for (int K = 1; K <= 8; ++K) {
+            if (!best.empty() && (int)best.size() <= target) break;
+            std::vector<std::vector<int>> steps;
+            std::vector<int> rem(n), cnt(n_idx);
+            for (int q = 0; q < n; ++q) rem[q] = q;
+            while (!rem.empty()) {
+                std::fill(cnt.begin(), cnt.end(), 0);
+                int rc[8] = {0, 0, 0, 0, 0, 0, 0, 0}, re[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                std::vector<int> st, rest;
+                for (int x : rem) {
+                    const CherryLane& L = ch[x];
+                    bool ok = st.size() < 32 && cnt[L.c] < K && cnt[L.e[0]] < K && (L.e[1] < 0 || cnt[L.e[1]] < K);
+                    if (ok && capped) {
+                        int ne[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                        ne[L.e[0] & 7]++;
+                        if (L.e[1] >= 0) ne[L.e[1] & 7]++;
+                        ok = rc[L.c & 7] < 4;
+                        for (int r = 0; r < 8 && ok; ++r) ok = re[r] + ne[r] <= 8;
+                    }
+                    if (!ok) {
+                        rest.push_back(x);
+                        continue;
+                    }
+                    st.push_back(x);
+                    cnt[L.c]++;
+                    cnt[L.e[0]]++;
+                    if (L.e[1] >= 0) cnt[L.e[1]]++;
+                    rc[L.c & 7]++;
+                    re[L.e[0] & 7]++;
+                    if (L.e[1] >= 0) re[L.e[1] & 7]++;
+                }
+                steps.push_back(std::move(st));
+                rem.swap(rest);
+            }
+            if (best.empty() || steps.size() < best.size()) {
+                best = std::move(steps);
+                bestK = K;
+            }
+        }
+        if ((int)best.size() <= target) break;
+    }
+    S.steps = (int)best.size();
+    S.slots = bestK;
+    if (S.steps > max_steps) return S;
+    S.lane.assign((size_t)S.steps * 32, CherryLane{});
+    // (3) placement: one local search over all positions (swaps within and across
+    // steps that keep every step within K targets per atom, and end flips)
+    const int NP = S.steps * 32, K = bestK;
+    std::vector<const CherryLane*> pos(NP, nullptr);
+    std::vector<uint8_t> flip(NP, 0);
+    std::vector<int> cnt((size_t)S.steps * n_idx, 0);
+    for (int st = 0; st < S.steps; ++st)
+        for (size_t l = 0; l < best[st].size(); ++l) {
+            const CherryLane* L = &ch[best[st][l]];
+            pos[st * 32 + (int)l] = L;
+            cnt[(size_t)st * n_idx + L->c]++;
+            for (int k = 0; k < 2; ++k)
+                if (L->e[k] >= 0) cnt[(size_t)st * n_idx + L->e[k]]++;
+        }
+    std::vector<int> qc(NP / 8);
+    for (int g = 0; g < NP / 8; ++g) qc[g] = cherry_quarter_cost(&pos[8 * g], &flip[8 * g]);
+    auto fits = [&](int st, const CherryLane* in, const CherryLane* out) {  // K after swapping `out` for `in` in step st
+        if (!in) return true;
+        const int at[3] = {in->c, in->e[0], in->e[1]};
+        for (int k = 0; k < 3; ++k) {
+            if (at[k] < 0) continue;
+            int c = cnt[(size_t)st * n_idx + at[k]] + 1;
+            if (out && (out->c == at[k] || out->e[0] == at[k] || out->e[1] == at[k])) --c;
+            if (c > K) return false;
+        }
+        return true;
+    };
+    auto move_cnt = [&](int st, const CherryLane* L, int d) {
+        if (!L) return;
+        cnt[(size_t)st * n_idx + L->c] += d;
+        for (int k = 0; k < 2; ++k)
+            if (L->e[k] >= 0) cnt[(size_t)st * n_idx + L->e[k]] += d;
+    };
+    // greedy local search (moves that do not add wavefronts), half of the moves
+    // targeted at a lane on a conflicting bank group; 400k moves per step at effort 2
+    // (config 2: ~0.4 s of host time at upload), a tenth at effort 1
+    static const long imul = getenv("AD_CHERRY_ITERS") ? atol(getenv("AD_CHERRY_ITERS")) : 400000;
+    const long iters = (long)(effort >= 2 ? imul : effort == 1 ? imul / 10 : 0) * S.steps;
+    uint64_t rng = 0x9E3779B97F4A7C15ull;
+    int total = 0, floor_cost = 0;  // floor: 3 per quarter-warp holding a cherry
+    for (int g = 0; g < NP / 8; ++g) total += qc[g];
+    for (int st = 0; st < S.steps; ++st) floor_cost += 3 * (((int)best[st].size() + 7) / 8);
+    for (long it = 0; it < iters && total > floor_cost; ++it) {
+        rng ^= rng << 13; rng ^= rng >> 7; rng ^= rng << 17;
+        int a = (int)(rng % (uint64_t)NP);
+        const int b = (int)((rng >> 24) % (uint64_t)NP);
+        if ((rng >> 40) & 1) {  // targeted: a lane on a bank group that conflicts in its quarter-warp
+            const int g = a >> 3;
+            if (qc[g] > 3) {
+                int best_acc = -1, best_r = -1, mx = 1;
+                for (int acc = 0; acc < 3; ++acc) {
+                    int c8[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                    for (int l = 8 * g; l < 8 * g + 8; ++l) {
+                        if (!pos[l]) continue;
+                        const int row = acc == 0 ? pos[l]->c : pos[l]->e[(acc - 1) ^ flip[l]];
+                        if (row >= 0 && ++c8[row & 7] > mx) { mx = c8[row & 7]; best_acc = acc; best_r = row & 7; }
+                    }
+                }
+                if (best_acc >= 0) {
+                    const int start = (int)((rng >> 48) & 7);
+                    for (int k = 0; k < 8; ++k) {
+                        const int l = 8 * g + ((start + k) & 7);
+                        if (!pos[l]) continue;
+                        const int row = best_acc == 0 ? pos[l]->c : pos[l]->e[(best_acc - 1) ^ flip[l]];
+                        if (row >= 0 && (row & 7) == best_r) { a = l; break; }
+                    }
+                }
+            }
+        }
+        const int ga = a >> 3, gb = b >> 3;
+        if ((rng >> 50) % 4 == 0) {  // flip the ends of position a
+            if (!pos[a]) continue;
+            flip[a] ^= 1;
+            const int c = cherry_quarter_cost(&pos[8 * ga], &flip[8 * ga]);
+            if (c <= qc[ga]) { total += c - qc[ga]; qc[ga] = c; } else flip[a] ^= 1;
+            continue;
+        }
+        if (ga == gb || (!pos[a] && !pos[b])) continue;
+        const int sa = a >> 5, sb = b >> 5;
+        if (sa != sb && (!fits(sa, pos[b], pos[a]) || !fits(sb, pos[a], pos[b]))) continue;
+        std::swap(pos[a], pos[b]);
+        std::swap(flip[a], flip[b]);
+        const int ca = cherry_quarter_cost(&pos[8 * ga], &flip[8 * ga]);
+        const int cb = cherry_quarter_cost(&pos[8 * gb], &flip[8 * gb]);
+        if (ca + cb <= qc[ga] + qc[gb]) {
+            total += ca + cb - qc[ga] - qc[gb];
+            qc[ga] = ca;
+            qc[gb] = cb;
+            if (sa != sb) {  // pos[a] came from step sb, pos[b] from step sa
+                move_cnt(sa, pos[b], -1);
+                move_cnt(sa, pos[a], +1);
+                move_cnt(sb, pos[a], -1);
+                move_cnt(sb, pos[b], +1);
+            }
+        } else {
+            std::swap(pos[a], pos[b]);
+            std::swap(flip[a], flip[b]);
+        }
+    }
+    for (int st = 0; st < S.steps; ++st) {
+        std::vector<int> c(n_idx, 0);
+        for (int l = 0; l < 32; ++l) {
+            CherryLane& o = S.lane[(size_t)st * 32 + l];
+            const CherryLane* src = pos[st * 32 + l];
+            if (!src) continue;
+            o = *src;
+            if (flip[st * 32 + l]) {
+                std::swap(o.e[0], o.e[1]);
+                std::swap(o.p[0], o.p[1]);
+            }
+            o.kc = c[o.c]++;
+            for (int k = 0; k < 2; ++k) o.ke[k] = o.e[k] >= 0 ? c[o.e[k]]++ : -1;
+        }
+    }
+    return S;
+}
+
+// Records of a cherry schedule (layout: ad_internal.h pka / pkb / pkc, kernel:
+// intra_cherry).  Empty ends and lanes get a zero-charge X row and a spare
+// gradient row in the bank group least used by that access in their
+// quarter-warp (distinct groups within a lane).
+struct CherryRecords {
+    std::vector<uint4> a;
+    std::vector<float4> b, c;
+};
+CherryRecords pack_cherries(const CherrySchedule& S, int npad, int ws_g, const std::vector<int>& ptp,
+                            const std::vector<float4>& tp, const std::vector<float>& pdsv) {
+    CherryRecords R;
+    const size_t n = (size_t)S.steps * 32;
+    R.a.resize(n);
+    R.b.resize(n);
+    R.c.resize(n);
+    const int K = S.slots;
+    auto xoff = [&](int row) { return (uint32_t)(16 * row); };
+    auto goff = [&](int row, int k) { return (uint32_t)(ws_g + 16 * (k * npad + row)); };
+    for (size_t q0 = 0; q0 < n; q0 += 8) {  // one quarter-warp
+        int cnt[3][8] = {};
+        for (size_t q = q0; q < q0 + 8; ++q) {
+            const CherryLane& L = S.lane[q];
+            if (L.c < 0) continue;
+            cnt[0][L.c & 7]++;
+            for (int k = 0; k < 2; ++k)
+                if (L.e[k] >= 0) cnt[1 + k][L.e[k] & 7]++;
+        }
+        for (size_t q = q0; q < q0 + 8; ++q) {
+            const CherryLane& L = S.lane[q];
+            uint32_t w[3];
+            unsigned taken = 0;  // bank groups of this lane's dummy rows (distinct positions)
+            auto dummy = [&](int acc) {
+                int r = -1;
+                for (int x = 0; x < 8; ++x)
+                    if (!(taken >> x & 1u) && (r < 0 || cnt[acc][x] < cnt[acc][r])) r = x;
+                taken |= 1u << r;
+                cnt[acc][r]++;
+                return xoff(npad + r) | (goff(r, K) << 16);
+            };
+            w[0] = L.c >= 0 ? xoff(L.c) | (goff(L.c, L.kc) << 16) : dummy(0);
+            float4 co[2];
+            float dsv[2];
+            for (int k = 0; k < 2; ++k) {
+                if (L.c >= 0 && L.e[k] >= 0) {
+                    w[1 + k] = xoff(L.e[k]) | (goff(L.e[k], L.ke[k]) << 16);
+                    const float4 t = tp[ptp[L.p[k]]];
+                    co[k] = make_float4(t.x, t.y, t.w > 8.f ? -t.z : t.z, 0.f);  // sign bit: 12-10 pair
+                    dsv[k] = pdsv[L.p[k]];
+                } else {
+                    w[1 + k] = dummy(1 + k);
+                    co[k] = make_float4(0.f, 0.f, 1.f, 0.f);
+                    dsv[k] = 0.f;
+                }
+            }
+            uint32_t ud;
+            memcpy(&ud, &dsv[0], 4);
+            R.a[q] = make_uint4(w[0], w[1], w[2], ud);
+            R.b[q] = make_float4(co[0].x, co[0].y, co[0].z, dsv[1]);
+            R.c[q] = make_float4(co[1].x, co[1].y, co[1].z, 0.f);
+        }
+    }
+    return R;
+}
+
 // Owner-computes list: every contributor pair (i, j) becomes two directed
 // entries (i <- j, primary) and (j <- i); entries are grouped by owner atom and
 // the concatenated list is cut into 32 equal slices (lane l takes entries
@@ -885,7 +1232,7 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
     if (!ctx) return fail(AD_ERR_OOM, "host allocation failed");
     ctx->device = cuda_device;
     if (const char* m = getenv("AD_PAIRS_SMEM_MAX")) ctx->pairs_smem_max = atoi(m);
-    if (const char* m = getenv("AD_PK_SMEM_MAX")) ctx->pk_smem_max = atoi(m);  // 0: no packed schedules (A/B)
+    if (const char* m = getenv("AD_PK_SMEM_MAX")) ctx->pk_smem_max = atoi(m);  // 0: no cherry schedules (A/B)
     if (const char* m = getenv("AD_INTRA_MODE"))
         ctx->intra_mode = strcmp(m, "owner") == 0 ? INTRA_OWNER : strcmp(m, "hybrid") == 0 ? INTRA_HYBRID : INTRA_SCATTER;
     cudaError_t e = cudaSetDevice(cuda_device);
@@ -1125,6 +1472,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     for (int k = 0; k < N; ++k) slot[k] = k;
     Schedule sch;
     OwnerList own;
+    CherrySchedule cs;
+    bool cherry = false;
     if (mode == INTRA_OWNER) {
         own = build_owner(N, pi, pj, ptp, pd);
         if (own.C * 32 > 65535) return fail(AD_ERR_LIMIT, "too many owner chunks");
@@ -1149,7 +1498,29 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             si[q] = slot[pi[q]];
             sj[q] = slot[pj[q]];
         }
-        sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
+        // the cherry schedule when it fits shared memory (records + the baseline's
+        // plain list) and its row offsets fit 16 bits; else the pair-step schedule
+        if (ctx->pk_smem_max > 0 && P > 0) {
+            const int max_steps = std::min(ctx->pairs_smem_max / (kPairsPerStep * 12), ctx->pk_smem_max / (kLanes * 48));
+            cs = schedule_cherries(npad_of(N), si, sj, ctx->sched_effort, max_steps);
+            const WarpScratch w = warp_scratch_layout(N, T, cs.slots, 0);
+            cherry = cs.steps <= max_steps && w.g + 16 * (npad_of(N) * (cs.slots + 1)) <= 0xffff;
+        }
+        if (cherry) {
+            // the paper-style baseline reads every pair once from the plain list
+            // (entries past P are empty: slot field = K)
+            sch.rounds = cs.steps;
+            sch.slots = cs.slots;
+            sch.rec.assign((size_t)cs.steps * kPairsPerStep, (uint32_t)cs.slots << 16);
+            sch.dsv.assign((size_t)cs.steps * kPairsPerStep * 2, 0.f);
+            for (int q = 0; q < P; ++q) {
+                sch.rec[q] = (uint32_t)si[q] | ((uint32_t)sj[q] << 8) | ((uint32_t)ptp[q] << 24);
+                sch.dsv[2 * q] = pd[q];
+                sch.dsv[2 * q + 1] = pcq[q];
+            }
+        } else {
+            sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
+        }
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -1227,36 +1598,16 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     const int32_t pair_bytes = (int32_t)B.buf.size() - H.off_prec;
     H.pairs_gmem = pair_bytes > ctx->pairs_smem_max ? 1 : 0;
     const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
-    // packed schedule (see ad_internal.h): scatter mode, schedule in shared memory,
-    // every row byte offset below 64 KiB
-    const int n_places = sch.rounds * kPairsPerStep;
-    const bool packed = mode == INTRA_SCATTER && !H.pairs_gmem && n_places > 0 &&
-                        n_places * 24 <= ctx->pk_smem_max && ws.g + 16 * (H.n_pad * (sch.slots + 1)) <= 0xffff;
+    // cherry schedule records (ad_internal.h pka / pkb / pkc): staged by the warp
+    // engine only (the baseline stages [0, off_pk))
     H.off_pk = 0;
+    if (cherry && H.pairs_gmem) return fail(AD_ERR_STATE, "internal: cherry schedule outside shared memory");
     const int32_t base_bytes = (int32_t)B.buf.size();
-    if (packed) {
-        std::vector<uint4> pka(n_places);
-        std::vector<float2> pkb(n_places);
-        const uint32_t npad = (uint32_t)H.n_pad;
-        for (int q = 0; q < n_places; ++q) {
-            const uint32_t rec = sch.rec[q];
-            const uint32_t i = rec & 0xffu, j = (rec >> 8) & 0xffu, si = (rec >> 16) & 0xfu, sj = (rec >> 20) & 0xfu;
-            const uint32_t gi = (uint32_t)ws.g + 16u * (si * npad + i);
-            const uint32_t gj = (uint32_t)ws.g + 16u * (sj * npad + j);
-            if ((int)si == sch.slots) {  // empty place: the zero-charge rows, zero coefficients, spare row
-                pka[q] = make_uint4((16u * npad) | ((16u * (npad + 1)) << 16), gi | (gj << 16), 0u, 0u);
-                pkb[q] = make_float2(0.f, 1.f);
-                continue;
-            }
-            const float4 c = tp[rec >> 24];
-            uint32_t ud, ua;
-            memcpy(&ud, &sch.dsv[2 * q], 4);
-            memcpy(&ua, &c.x, 4);
-            pka[q] = make_uint4((16u * i) | ((16u * j) << 16), gi | (gj << 16), ud, ua);
-            pkb[q] = make_float2(c.y, c.w > 8.f ? -c.z : c.z);  // sign bit = 12-10 (H-bond) pair
-        }
-        H.off_pk = B.put(pka.data(), sizeof(uint4) * pka.size());
-        B.put(pkb.data(), sizeof(float2) * pkb.size());
+    if (cherry) {
+        const CherryRecords cr = pack_cherries(cs, H.n_pad, ws.g, ptp, tp, pd);
+        H.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
+        B.put(cr.b.data(), sizeof(float4) * cr.b.size());
+        B.put(cr.c.data(), sizeof(float4) * cr.c.size());
     }
     H.blob_bytes = (int32_t)B.buf.size();
     if (const char* dump = getenv("AD_DUMP_SCHEDULE")) {  // debugging aid: raw schedule records
@@ -1792,6 +2143,40 @@ int32_t adx_debug_schedule(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
     *out_slots = s.slots;
     if (out_rec)
         for (int q = 0; q < std::min<int>(cap, (int)s.rec.size()); ++q) out_rec[q] = s.rec[q];
+    return AD_OK;
+}
+
+// Host-only inspection hook (not part of include/ad.h; no GPU needed): the cherry
+// schedule of a pair list (storage rows from balance_slots, as at upload).  out
+// receives [steps*32][8] int32: centre, end0, end1 (rows), pair0, pair1 (ids),
+// slot of centre / end0 / end1 (-1 = empty).
+int32_t adx_debug_cherries(int32_t n_atoms, int32_t n_pairs, const int32_t* pairs, int32_t effort, int32_t* out_steps,
+                           int32_t* out_slots, int32_t* out, int32_t cap_lanes, int32_t* out_atom_slot) {
+    if (n_atoms < 1 || n_atoms > AD_MAX_ATOMS || n_pairs < 0 || (n_pairs && !pairs) || !out_steps || !out_slots)
+        return fail(AD_ERR_INVALID_ARG, "bad arguments");
+    std::vector<int> pi(n_pairs), pj(n_pairs);
+    for (int q = 0; q < n_pairs; ++q) {
+        pi[q] = pairs[2 * q];
+        pj[q] = pairs[2 * q + 1];
+        if (pi[q] < 0 || pi[q] >= n_atoms || pj[q] < 0 || pj[q] >= n_atoms || pi[q] == pj[q])
+            return fail(AD_ERR_INVALID_ARG, "bad pair %d", q);
+    }
+    const std::vector<int> slot = balance_slots(n_atoms, pi, pj);
+    for (int q = 0; q < n_pairs; ++q) {
+        pi[q] = slot[pi[q]];
+        pj[q] = slot[pj[q]];
+    }
+    if (out_atom_slot)
+        for (int a = 0; a < n_atoms; ++a) out_atom_slot[a] = slot[a];
+    const CherrySchedule S = schedule_cherries(npad_of(n_atoms), pi, pj, effort);
+    *out_steps = S.steps;
+    *out_slots = S.slots;
+    if (out)
+        for (int q = 0; q < std::min<int>(cap_lanes, (int)S.lane.size()); ++q) {
+            const CherryLane& L = S.lane[q];
+            const int v[8] = {L.c, L.e[0], L.e[1], L.p[0], L.p[1], L.kc, L.ke[0], L.ke[1]};
+            for (int k = 0; k < 8; ++k) out[8 * q + k] = v[k];
+        }
     return AD_OK;
 }
 

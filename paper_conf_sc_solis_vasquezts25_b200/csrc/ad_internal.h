@@ -24,15 +24,9 @@
 //            partial slots k*32+lane that belong to atom a)
 //   tp      float4 [nt*nt*8] cA, cB, r0, n (m == 12); 8 copies per entry (index t*8+c),
 //                           lane l reads copy l%8 -> conflict-free 128-bit lookups
-//   pka     u32x4  [R*64]   (packed schedule, off_pk != 0: INTRA_SCATTER with the schedule
-//                           in shared memory) the same places as prec, pre-decoded:
-//                           {X row byte offsets i | j<<16, gradient row byte offsets
-//                           (per-warp scratch relative, slot * npad + row) i | j<<16,
-//                           dsv bits, cA bits}
-//   pkb     float2 [R*64]   cB, r0 with the sign bit set for n = 10 (H-bond).  The
-//                           kernel forms coeff_el q_i q_j from the X rows' charges.
-//                           Empty places read the two zero-charge X rows with
-//                           cA = cB = dsv = 0: their E and dE/dr are exactly 0.
+//   pka     u32x4  [R*32]   (cherry schedule, off_pk != 0: INTRA_SCATTER with the schedule
+//   pkb     f32x4  [R*32]   in shared memory; R = n_rounds cherry steps of 32 lanes, each lane
+//   pkc     f32x4  [R*32]   two pairs sharing a centre atom) -- see intra_cherry in ad_kernels.cuh
 //           The warp engine stages the whole blob; the paper-style baseline stages
 //           [0, off_pk) (prec / pdsv / tp), its footprint unchanged.
 //
@@ -123,7 +117,7 @@ struct GridDev {
 
 // Per-warp scratch layout (offsets in bytes from the warp's slice; 16-aligned).
 struct WarpScratch {
-    int32_t x;      // float4 [Npad+2]      world coords + charge (+ 2 zero-charge rows)
+    int32_t x;      // float4 [Npad+8]      world coords + charge (+ 8 zero-charge rows)
     int32_t g;      // float4 [K][Npad]+8   atom gradient accumulators (slot 0 seeded with inter) + 8 spare
     int32_t w;      // float4 [Npad+1][2]   W staging (TC engines only)
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
@@ -143,9 +137,9 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     const int32_t npad = (n_atoms + 7) & ~7;
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
     int32_t o = 0;
-    // X rows + two zero-charge rows (positions (0,0,0), (1,0,0)) that the empty
-    // places of packed schedules read
-    s.x = o;     o += 16 * (npad + 2);
+    // X rows + 8 zero-charge rows (positions (r,0,0), bank group r) that the empty
+    // ends of cherry schedules read
+    s.x = o;     o += 16 * (npad + 8);
     // rows of npad float4 (slot k of atom a at k * npad + a) + the start of a spare
     // row K: empty schedule places only ever target K * npad + (0..7)
     s.g = o;     o += 16 * npad * n_slots + 16 * 8;
