@@ -54,7 +54,8 @@ int32_t fail(int32_t code, const char* fmt, ...) {
     } while (0)
 
 struct LigSlot {
-    unsigned char* d_blob = nullptr;
+    unsigned char* d_blob = nullptr;  // the warp engines' blob
+    unsigned char* d_base = nullptr;  // the paper-style baseline's (== d_blob unless cherries)
     int32_t blob_bytes = 0;      // staged by the warp engine
     int32_t base_bytes = 0;      // staged by the paper-style baseline
     int32_t scratch_bytes = 0;   // per warp (TC engine)
@@ -125,7 +126,8 @@ int32_t sync_ligtab(ad_context* ctx, int only = -1) {
     const int n = (int)ctx->ligs.size();
     if (only >= 0 && only < ctx->ligtab_cap) {
         const LigSlot& L = ctx->ligs[only];
-        const LigDev e{L.live ? L.d_blob : nullptr, L.blob_bytes, L.scratch_bytes, L.scratch_simt, L.base_bytes};
+        const LigDev e{L.live ? L.d_blob : nullptr, L.blob_bytes, L.scratch_bytes, L.scratch_simt, L.base_bytes,
+                       L.live ? L.d_base : nullptr};
         CUDA_TRY(cudaMemcpy(ctx->d_ligtab + only, &e, sizeof(LigDev), cudaMemcpyHostToDevice));
         return AD_OK;
     }
@@ -141,7 +143,8 @@ int32_t sync_ligtab(ad_context* ctx, int only = -1) {
     std::vector<LigDev> h(n);
     for (int i = 0; i < n; ++i)
         h[i] = LigDev{ctx->ligs[i].live ? ctx->ligs[i].d_blob : nullptr, ctx->ligs[i].blob_bytes,
-                      ctx->ligs[i].scratch_bytes, ctx->ligs[i].scratch_simt, ctx->ligs[i].base_bytes};
+                      ctx->ligs[i].scratch_bytes, ctx->ligs[i].scratch_simt, ctx->ligs[i].base_bytes,
+                      ctx->ligs[i].live ? ctx->ligs[i].d_base : nullptr};
     if (n) CUDA_TRY(cudaMemcpy(ctx->d_ligtab, h.data(), sizeof(LigDev) * n, cudaMemcpyHostToDevice));
     return AD_OK;
 }
@@ -1255,8 +1258,10 @@ int32_t ad_context_destroy(ad_context* ctx) {
     if (!ctx) return AD_OK;
     cudaSetDevice(ctx->device);
     cudaDeviceSynchronize();
-    for (auto& l : ctx->ligs)
+    for (auto& l : ctx->ligs) {
+        if (l.d_base && l.d_base != l.d_blob) cudaFree(l.d_base);
         if (l.d_blob) cudaFree(l.d_blob);
+    }
     if (ctx->d_tmap) cudaFree(ctx->d_tmap);
     if (ctx->d_ed) cudaFree(ctx->d_ed);
     if (ctx->d_ligtab) cudaFree(ctx->d_ligtab);
@@ -1498,29 +1503,19 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             si[q] = slot[pi[q]];
             sj[q] = slot[pj[q]];
         }
-        // the cherry schedule when it fits shared memory (records + the baseline's
-        // plain list) and its row offsets fit 16 bits; else the pair-step schedule
+        // the cherry schedule when it fits shared memory (its records and the prec
+        // list) and its row offsets fit 16 bits; else the pair-step schedule
         if (ctx->pk_smem_max > 0 && P > 0) {
             const int max_steps = std::min(ctx->pairs_smem_max / (kPairsPerStep * 12), ctx->pk_smem_max / (kLanes * 48));
             cs = schedule_cherries(npad_of(N), si, sj, ctx->sched_effort, max_steps);
             const WarpScratch w = warp_scratch_layout(N, T, cs.slots, 0);
             cherry = cs.steps <= max_steps && w.g + 16 * (npad_of(N) * (cs.slots + 1)) <= 0xffff;
         }
-        if (cherry) {
-            // the paper-style baseline reads every pair once from the plain list
-            // (entries past P are empty: slot field = K)
-            sch.rounds = cs.steps;
-            sch.slots = cs.slots;
-            sch.rec.assign((size_t)cs.steps * kPairsPerStep, (uint32_t)cs.slots << 16);
-            sch.dsv.assign((size_t)cs.steps * kPairsPerStep * 2, 0.f);
-            for (int q = 0; q < P; ++q) {
-                sch.rec[q] = (uint32_t)si[q] | ((uint32_t)sj[q] << 8) | ((uint32_t)ptp[q] << 24);
-                sch.dsv[2 * q] = pd[q];
-                sch.dsv[2 * q + 1] = pcq[q];
-            }
-        } else {
-            sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
-        }
+        // the prec list (the paper-style baseline's pairs; the warp engine's schedule
+        // when it runs no cherries) is the pair-step schedule either way, so the
+        // baseline is the same program with or without cherries
+        sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
+        if (cherry && (int64_t)(sch.rec.size() + sch.dsv.size()) * 4 > ctx->pairs_smem_max) cherry = false;
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -1557,7 +1552,9 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
 
     LigHeader H{};
     H.n_atoms = N; H.n_tors = T; H.n_pairs = P; H.n_types = nt;
-    H.n_rounds = sch.rounds; H.n_slots = sch.slots; H.n_chain = (int)chain.size();
+    H.n_rounds = sch.rounds;  // per blob below
+    H.n_slots = sch.slots;
+    H.n_chain = (int)chain.size();
     H.n_pad = npad_of(N);  // gradient-slot row stride
     H.intra_mode = mode;
     H.n_entries = own.E;
@@ -1575,41 +1572,10 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     H.ff[FF_DS_EXP2] = (float)(-1.4426950408889634 / (2.0 * sig * sig));
     H.ff[FF_INV_S2] = (float)(1.0 / (sig * sig));
     H.ff[FF_W_OUT] = F.w_out;
-    BlobBuilder B;
-    B.put(&H, sizeof(H));
-    H.off_atoms = B.put(atoms.data(), sizeof(float4) * N);
-    H.off_info = B.put(info.data(), sizeof(int2) * N);
-    H.off_tors = B.put(tors.data(), sizeof(float4) * 2 * T);
-    H.off_tinfo = B.put(tinfo.data(), sizeof(int4) * T);
-    H.off_chain = B.put(chain.data(), chain.size());
-    H.off_mask = B.put(mask.data(), sizeof(uint2) * N);
-    // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
-    // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
-    std::vector<float4> tp8(tp.size() * AD_TP_COPIES);
-    for (size_t t = 0; t < tp.size(); ++t)
-        for (int c = 0; c < AD_TP_COPIES; ++c) tp8[t * AD_TP_COPIES + c] = tp[t];
-    H.off_tp = B.put(tp8.data(), sizeof(float4) * tp8.size());
-    H.off_comb = B.put(own.comb.data(), sizeof(int2) * own.comb.size());
-    H.off_combidx = B.put(own.combidx.data(), sizeof(uint16_t) * own.combidx.size());
-    // the pair schedule goes last: large schedules stay in global memory (read
-    // through L1, one copy per SM) instead of being staged into every CTA
-    H.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
-    H.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
-    const int32_t pair_bytes = (int32_t)B.buf.size() - H.off_prec;
-    H.pairs_gmem = pair_bytes > ctx->pairs_smem_max ? 1 : 0;
-    const WarpScratch ws = warp_scratch_layout(N, T, sch.slots, own.C);
-    // cherry schedule records (ad_internal.h pka / pkb / pkc): staged by the warp
-    // engine only (the baseline stages [0, off_pk))
-    H.off_pk = 0;
-    if (cherry && H.pairs_gmem) return fail(AD_ERR_STATE, "internal: cherry schedule outside shared memory");
-    const int32_t base_bytes = (int32_t)B.buf.size();
-    if (cherry) {
-        const CherryRecords cr = pack_cherries(cs, H.n_pad, ws.g, ptp, tp, pd);
-        H.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
-        B.put(cr.b.data(), sizeof(float4) * cr.b.size());
-        B.put(cr.c.data(), sizeof(float4) * cr.c.size());
-    }
-    H.blob_bytes = (int32_t)B.buf.size();
+    // Two blobs when the warp engine runs a cherry schedule: the warp engine's (tables +
+    // cherry records; no pair-step list, no type-pair table) and the paper-style
+    // baseline's (tables + type-pair table + the pair-step list), so neither stages
+    // bytes it never reads.  Otherwise one blob serves both engines.
     if (const char* dump = getenv("AD_DUMP_SCHEDULE")) {  // debugging aid: raw schedule records
         if (FILE* f = fopen(dump, "ab")) {
             const int32_t hdr[4] = {N, sch.rounds, sch.slots, H.n_pad};
@@ -1618,30 +1584,96 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             fclose(f);
         }
     }
-    H.stage_bytes = H.pairs_gmem ? H.off_prec : H.blob_bytes;
-    H.scratch_bytes = ws.bytes;
-    H.ws_g = ws.g; H.ws_w = ws.w; H.ws_d = ws.d; H.ws_trig = ws.trig;
-    H.ws_tw = ws.tw; H.ws_genes = ws.genes; H.ws_part = ws.part;
-    memcpy(B.buf.data(), &H, sizeof(H));
+    if (cherry && (int64_t)(sch.rec.size() + sch.dsv.size()) * 4 > ctx->pairs_smem_max)
+        return fail(AD_ERR_STATE, "internal: cherry schedule with a global-memory prec list");
+    struct Built {
+        std::vector<unsigned char> buf;
+        LigHeader h;
+        WarpScratch ws;
+    };
+    auto build_blob = [&](bool warp_cherry) {
+        Built o;
+        LigHeader& h = o.h;
+        h = H;
+        h.n_rounds = warp_cherry ? cs.steps : sch.rounds;
+        h.n_slots = warp_cherry ? cs.slots : sch.slots;
+        h.base_rounds = sch.rounds;
+        h.base_slots = sch.slots;
+        BlobBuilder B;
+        B.put(&h, sizeof(h));
+        h.off_atoms = B.put(atoms.data(), sizeof(float4) * N);
+        h.off_info = B.put(info.data(), sizeof(int2) * N);
+        h.off_tors = B.put(tors.data(), sizeof(float4) * 2 * T);
+        h.off_tinfo = B.put(tinfo.data(), sizeof(int4) * T);
+        h.off_chain = B.put(chain.data(), chain.size());
+        h.off_mask = B.put(mask.data(), sizeof(uint2) * N);
+        h.off_comb = B.put(own.comb.data(), sizeof(int2) * own.comb.size());
+        h.off_combidx = B.put(own.combidx.data(), sizeof(uint16_t) * own.combidx.size());
+        o.ws = warp_scratch_layout(N, T, h.n_slots, own.C);
+        if (warp_cherry) {
+            // cherry records (ad_internal.h pka / pkb / pkc), staged with the tables
+            const CherryRecords cr = pack_cherries(cs, h.n_pad, o.ws.g, ptp, tp, pd);
+            h.off_tp = h.off_prec = h.off_pdsv = 0;
+            h.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
+            B.put(cr.b.data(), sizeof(float4) * cr.b.size());
+            B.put(cr.c.data(), sizeof(float4) * cr.c.size());
+            h.pairs_gmem = 0;
+            h.blob_bytes = h.stage_bytes = (int32_t)B.buf.size();
+        } else {
+            // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
+            // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
+            std::vector<float4> tp8(tp.size() * AD_TP_COPIES);
+            for (size_t t = 0; t < tp.size(); ++t)
+                for (int c = 0; c < AD_TP_COPIES; ++c) tp8[t * AD_TP_COPIES + c] = tp[t];
+            h.off_tp = B.put(tp8.data(), sizeof(float4) * tp8.size());
+            // the pair schedule goes last: large schedules stay in global memory (read
+            // through L1, one copy per SM) instead of being staged into every CTA
+            h.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
+            h.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
+            h.off_pk = 0;
+            h.pairs_gmem = (int32_t)B.buf.size() - h.off_prec > ctx->pairs_smem_max ? 1 : 0;
+            h.blob_bytes = (int32_t)B.buf.size();
+            h.stage_bytes = h.pairs_gmem ? h.off_prec : h.blob_bytes;
+        }
+        h.scratch_bytes = o.ws.bytes;
+        h.ws_g = o.ws.g; h.ws_w = o.ws.w; h.ws_d = o.ws.d; h.ws_trig = o.ws.trig;
+        h.ws_tw = o.ws.tw; h.ws_genes = o.ws.genes; h.ws_part = o.ws.part;
+        memcpy(B.buf.data(), &h, sizeof(h));
+        o.buf = std::move(B.buf);
+        return o;
+    };
+    const Built base = build_blob(false);
+    Built warp;
+    if (cherry) warp = build_blob(true);
+    const Built& W = cherry ? warp : base;
 
     std::lock_guard<std::mutex> lock(ctx->mu);
     if (int32_t rc = set_device(ctx)) return rc;
     LigSlot s;
-    s.blob_bytes = H.stage_bytes;  // shared-memory bytes staged per CTA (warp engine)
-    s.base_bytes = H.pairs_gmem ? H.off_prec : base_bytes;  // paper-style baseline: no packed schedule
-    s.scratch_bytes = ws.bytes;
-    s.scratch_simt = ws.bytes_simt;
+    s.blob_bytes = W.h.stage_bytes;     // shared-memory bytes staged per CTA (warp engine)
+    s.base_bytes = base.h.stage_bytes;  // ... (paper-style baseline)
+    s.scratch_bytes = W.ws.bytes;
+    s.scratch_simt = W.ws.bytes_simt;
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
     memcpy(s.ff, H.ff, sizeof(s.ff));
-    CUDA_TRY(cudaMalloc(&s.d_blob, B.buf.size()));
-    CUDA_TRY(cudaMemcpy(s.d_blob, B.buf.data(), B.buf.size(), cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMalloc(&s.d_blob, W.buf.size()));
+    CUDA_TRY(cudaMemcpy(s.d_blob, W.buf.data(), W.buf.size(), cudaMemcpyHostToDevice));
+    s.d_base = s.d_blob;
+    if (cherry) {
+        if (cudaMalloc(&s.d_base, base.buf.size()) != cudaSuccess) {
+            cudaFree(s.d_blob);
+            return fail(AD_ERR_OOM, "ligand blob allocation failed");
+        }
+        CUDA_TRY(cudaMemcpy(s.d_base, base.buf.data(), base.buf.size(), cudaMemcpyHostToDevice));
+    }
     s.live = true;
     // the lowest free id (ids of freed ligands are reused), else a new one
     int id = 0;
     while (id < (int)ctx->ligs.size() && ctx->ligs[id].live) ++id;
     if (id >= AD_MAX_LIGANDS) {
+        if (s.d_base != s.d_blob) cudaFree(s.d_base);
         cudaFree(s.d_blob);
         return fail(AD_ERR_LIMIT, "too many ligands");
     }
@@ -1658,6 +1690,7 @@ int32_t ad_free_ligand(ad_context* ctx, ad_ligand_id lig) {
         return fail(AD_ERR_INVALID_ARG, "bad ligand id %d", lig);
     if (int32_t rc = set_device(ctx)) return rc;
     CUDA_TRY(cudaDeviceSynchronize());
+    if (ctx->ligs[lig].d_base != ctx->ligs[lig].d_blob) cudaFree(ctx->ligs[lig].d_base);
     cudaFree(ctx->ligs[lig].d_blob);
     ctx->ligs[lig] = LigSlot{};
     return sync_ligtab(ctx, lig);

@@ -82,8 +82,10 @@ struct alignas(16) LigHeader {
     int32_t n_entries, n_chunks, off_comb, off_combidx; // 96  (owner mode: E per lane, chunks per lane)
     int32_t pairs_gmem, stage_bytes, ws_g, ws_w;        // 112: schedule in global memory?, bytes staged to smem
     int32_t ws_d, ws_trig, ws_tw, ws_genes;             // 128  per-warp scratch offsets (WarpScratch, ws_x = 0),
-    int32_t ws_part, off_pk, reserved1, reserved2;      // 144  precomputed so kernels reload, not recompute, them;
-                                                        //      off_pk: packed schedule (0 = none)
+    int32_t ws_part, off_pk, base_rounds, base_slots;   // 144  precomputed so kernels reload, not recompute, them;
+                                                        //      off_pk: cherry records (0 = none); base_*: steps
+                                                        //      and slots of the prec list (= n_rounds / n_slots
+                                                        //      unless the warp engine runs a cherry schedule)
     float ff[FF_N];                                     // 208
 };
 static_assert(sizeof(LigHeader) == 208, "header size");
@@ -94,7 +96,8 @@ struct LigDev {
     int32_t blob_bytes;         // bytes the warp engine stages into shared memory (header .. tables [.. schedule])
     int32_t scratch_bytes;      // per-warp scratch, TC engine
     int32_t scratch_simt;       // per-warp scratch, SIMT engine (no D tile)
-    int32_t base_bytes;         // bytes the paper-style baseline stages (no packed schedule)
+    int32_t base_bytes;         // bytes the paper-style baseline stages from base_blob
+    const unsigned char* base_blob;  // the baseline's blob (== blob unless the warp engine runs cherries)
 };
 
 // Grid in device memory, x-pair layout:
