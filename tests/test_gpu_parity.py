@@ -479,3 +479,30 @@ def test_alternative_intra_modes(ad, cfg2, mode, monkeypatch):
                      f"cfg2 {mode} LS")
     finally:
         c.close()
+
+
+@pytest.mark.parametrize("smooth", [0.5, 0.0])
+def test_cherry_schedule_shapes(ctx, smooth):
+    """The cherry pair loop (shared-memory schedules) on ligands that exercise its
+    corner cases: a tiny ligand (empty lanes, singles), odd pair counts, 33-64 atoms
+    (second atoms taken from the root fragment), no torsions; and smooth = 0 (no
+    flat band: empty ends must read two distinct zero-charge rows, or their zero
+    coefficients would multiply 1/0).  Score with gradients + a short shadowed LS."""
+    grid = synth.make_grid(91, 40, synth.TYPESETS[8], 600)
+    ff = synth.FFParams(smooth=smooth)
+    _uploaded.clear()
+    ctx.upload_grid(grid)
+    for seed, n_atoms, n_tors in [(11, 9, 1), (12, 23, 5), (13, 33, 6), (14, 50, 12), (15, 30, 0)]:
+        L = synth.make_ligand(seed, n_atoms, n_tors, 8)
+        lid = ctx.upload_ligand(L, ff)
+        genes = synth.make_genotypes(seed, 96, n_tors, grid)
+        g = torch.from_numpy(genes).cuda()
+        E, G, _ = ctx.score(lid, g)
+        torch.cuda.synchronize()
+        check_scores(L, grid, ff, genes, E.cpu().numpy(), G.cpu().numpy(), f"cherry n={n_atoms} smooth={smooth}")
+        tr, bE, *_ = _ls(ctx, lid, genes[:16], "simt", 8)
+        assert np.all(np.isfinite(bE)) and np.all(bE == tr[:, :, 0].min(axis=1))
+        for it in (0, 7):  # the trace's energies are the oracle's energies of the traced genes
+            Eo, _, aux, _ = O.score(L, grid, ff, tr[:, it, 1:1 + genes.shape[1]])
+            assert np.all(energy_gate(tr[:, it, 0], Eo, energy_scale(aux)) | (aux[:, O.AUX_MARGIN_E] < KINK))
+    _uploaded.clear()
