@@ -62,6 +62,7 @@ struct LigSlot {
     int32_t scratch_simt = 0;    // per warp (SIMT engine)
     int32_t block_scratch = 0;   // per block (baseline)
     int32_t n_atoms = 0, n_tors = 0;
+    bool pkg = false;            // pre-decoded global-memory schedule (wide 128-register kernels)
     float ff[FF_N] = {};         // LigHeader::ff (kernel parameters of every launch)
     bool live = false;
 };
@@ -1613,7 +1614,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         if (warp_cherry) {
             // cherry records (ad_internal.h pka / pkb / pkc), staged with the tables
             const CherryRecords cr = pack_cherries(cs, h.n_pad, o.ws.g, ptp, tp, pd);
-            h.off_tp = h.off_prec = h.off_pdsv = 0;
+            h.off_tp = h.off_prec = h.off_pdsv = h.off_pkg = 0;
             h.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
             B.put(cr.b.data(), sizeof(float4) * cr.b.size());
             B.put(cr.c.data(), sizeof(float4) * cr.c.size());
@@ -1631,7 +1632,37 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             h.off_prec = B.put(sch.rec.data(), sizeof(uint32_t) * sch.rec.size());
             h.off_pdsv = B.put(sch.dsv.data(), sizeof(float) * sch.dsv.size());
             h.off_pk = 0;
+            h.off_pkg = 0;
             h.pairs_gmem = (int32_t)B.buf.size() - h.off_prec > ctx->pairs_smem_max ? 1 : 0;
+            static const bool pkg_on = !getenv("AD_PKG") || atoi(getenv("AD_PKG")) != 0;  // A/B knob
+            if (h.pairs_gmem && pkg_on && h.intra_mode == INTRA_SCATTER &&
+                o.ws.g + 16 * (h.n_pad * (h.n_slots + 1)) <= 0xffff) {
+                // pre-decoded places for the global-memory pair loop (intra_packed_gm),
+                // after the prec list (never staged; the baseline keeps reading prec)
+                const int n_places = (int)sch.rec.size();
+                const uint32_t npad = (uint32_t)h.n_pad;
+                std::vector<uint4> pka(n_places);
+                std::vector<float2> pkb(n_places);
+                for (int q = 0; q < n_places; ++q) {
+                    const uint32_t rec = sch.rec[q];
+                    const uint32_t i = rec & 0xffu, j = (rec >> 8) & 0xffu, si = (rec >> 16) & 0xfu, sj = (rec >> 20) & 0xfu;
+                    const uint32_t gi = (uint32_t)o.ws.g + 16u * (si * npad + i);
+                    const uint32_t gj = (uint32_t)o.ws.g + 16u * (sj * npad + j);
+                    if ((int)si == sch.slots) {  // empty place: zero-charge rows, zero coefficients, spare row
+                        pka[q] = make_uint4((16u * npad) | ((16u * (npad + 1)) << 16), gi | (gj << 16), 0u, 0u);
+                        pkb[q] = make_float2(0.f, 1.f);
+                        continue;
+                    }
+                    const float4 c = tp[rec >> 24];
+                    uint32_t ud, ua;
+                    memcpy(&ud, &sch.dsv[2 * q], 4);
+                    memcpy(&ua, &c.x, 4);
+                    pka[q] = make_uint4((16u * i) | ((16u * j) << 16), gi | (gj << 16), ud, ua);
+                    pkb[q] = make_float2(c.y, c.w > 8.f ? -c.z : c.z);  // sign bit = 12-10 (H-bond) pair
+                }
+                h.off_pkg = B.put(pka.data(), sizeof(uint4) * pka.size());
+                B.put(pkb.data(), sizeof(float2) * pkb.size());
+            }
             h.blob_bytes = (int32_t)B.buf.size();
             h.stage_bytes = h.pairs_gmem ? h.off_prec : h.blob_bytes;
         }
@@ -1657,6 +1688,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
+    s.pkg = W.h.off_pkg != 0 && 6 + T > 32;
     memcpy(s.ff, H.ff, sizeof(s.ff));
     CUDA_TRY(cudaMalloc(&s.d_blob, W.buf.size()));
     CUDA_TRY(cudaMemcpy(s.d_blob, W.buf.data(), W.buf.size(), cudaMemcpyHostToDevice));
@@ -1820,9 +1852,15 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     struct Cand { int w = 0, active = -1; double cost = 1e300; size_t sm_smem = 0; size_t smem = 0; WarpKernelFn k = nullptr; };
     Cand pick;
     static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
+    // ligands with pre-decoded global-memory schedules run the 128-register kernels,
+    // which alone carry that loop (config 3: 121.0 ms vs 130.6 ms on the 80-register
+    // kernels' record-decoding loop)
+    bool pkg = L.pkg;
+    if (p.pose_ligand) for_each_launch_ligand(ctx, [&](const LigSlot& o) { pkg |= o.pkg; });
     for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
         if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
+        if (!force && pkg && !v) continue;
         for (int w = 1; w <= 32; ++w) {
             if (req_warps > 0 && w != req_warps) continue;
             if (p.pose_ligand && ((w & (w - 1)) || w > 8)) continue;  // ad.h: ligand runs are multiples of 8

@@ -4,7 +4,7 @@
 // shared memory with a single TMA bulk copy (cp.async.bulk) and keeps for all
 // max_iters ADADELTA iterations.  Layout (offsets in LigHeader, bytes):
 //
-//   LigHeader                                   208 B
+//   LigHeader                                   224 B
 //   atoms   float4 [N]      reference x,y,z (A, DFS order), charge q
 //   info    int2   [N]      {map | type<<8 | chain_len<<16 | slot<<24, chain_start}; slot =
 //                           the atom's storage row in the per-pose X / gradient arrays
@@ -86,9 +86,10 @@ struct alignas(16) LigHeader {
                                                         //      off_pk: cherry records (0 = none); base_*: steps
                                                         //      and slots of the prec list (= n_rounds / n_slots
                                                         //      unless the warp engine runs a cherry schedule)
-    float ff[FF_N];                                     // 208
+    int32_t off_pkg, reserved1, reserved2, reserved3;   // 160  off_pkg: pre-decoded global-memory places (0 = none)
+    float ff[FF_N];                                     // 224
 };
-static_assert(sizeof(LigHeader) == 208, "header size");
+static_assert(sizeof(LigHeader) == 224, "header size");
 
 // Device table entry, one per uploaded ligand.
 struct LigDev {
