@@ -155,6 +155,22 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.sm), "sampler": getattr(self, "mode", None)}
 
 
+def load_co_bounds(engine, config):
+    """Issue and L1/shared data-pipe utilisation of the LS kernel from the committed
+    ncu --set full summary of the same workload (profiles/ncu_summary.json), if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        k = json.load(open(path)).get("ls_kernel", {}).get(f"config{config}_{engine}")
+        if not k or "issue_active_pct" not in k:
+            return None
+        return {"issue_active": k["issue_active_pct"] / 100.0, "l1tex_throughput": k["l1tex_throughput_pct"] / 100.0,
+                "warp_instructions_per_launch": k.get("warp_instructions"),
+                "shared_wavefronts_per_launch": k.get("shared_wavefronts"),
+                "source": f"profiles/ncu_{k['round']}.md ({k['report']}, ncu --set full)"}
+    except (OSError, ValueError, KeyError):
+        return None
+
+
 def load_traffic(engine, config):
     """dram bytes per launch of the LS kernel from a committed ncu --set full summary, if any."""
     path = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -522,7 +538,10 @@ def main():
                 "flops_per_eval": work["flops"], "mufu_per_eval": work["mufu"],
                 "mufu_frac": work["mufu"] * n * w.iters / kern_avg_s / (148 * 16 * 1965e6),
                 "l2_gather_gbs": work["l2_bytes"] * n * w.iters / kern_avg_s / 1e9,
-                "kernel_ms_avg": kern_avg_s * 1e3}
+                "kernel_ms_avg": kern_avg_s * 1e3,
+                # the units that actually bound the kernel: the FP32 flop model
+                # counts useful arithmetic only, issue slots and the L1/shared pipe saturate first
+                "co_bounds": load_co_bounds(args.engine, args.config)}
 
     # ---- CPU baseline (the oracle as it stands) + max |dE| vs the oracle ----
     cpu = None

@@ -59,6 +59,13 @@ def main():
             dw = float(s["dram__bytes_write.sum"][0]) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[
                 s["dram__bytes_write.sum"][1]]
             js["ls_kernel"][key] = {"dram_bytes_per_launch": dr + dw, "round": rnd, "report": os.path.basename(path)}
+            # the measured co-bounds of the kernel (bench.py roofline.co_bounds)
+            for name, metric in (("issue_active_pct", "smsp__issue_active.avg.pct_of_peak_sustained_active"),
+                                 ("l1tex_throughput_pct", "l1tex__throughput.avg.pct_of_peak_sustained_active"),
+                                 ("warp_instructions", "smsp__inst_executed.sum"),
+                                 ("shared_wavefronts", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")):
+                if metric in s:
+                    js["ls_kernel"][key][name] = float(s[metric][0])
         except (KeyError, ValueError):
             pass
     open(os.path.join(ROOT, "profiles", f"ncu_{rnd}.md"), "w").write("\n".join(lines) + "\n")
