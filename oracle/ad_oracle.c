@@ -137,12 +137,12 @@ static double gv(const ado_grid* G, int m, int x, int y, int z) {
  * inside : E = sum_c prod_k w_k(c) * (T_m + q E + |q| D)[corner c]  (trilinear)
  *          dE/dX = (1/h) d/du of the same interpolant (Z3)
  * outside: E = w_out * sum_k (u_k - c_k)^2, c = (n-1)/2, dE/dX = 2 w_out (u-c)/h (Z4).
- * abs_e / abs_g: magnitude sums for the Z18 tolerance (sum over every term of
- * |term| and of |d term/dX| component-wise).  margin_e / margin_g: distance
+ * abs_e: magnitude sum for the Z18 tolerance (sum over the weighted corner
+ * terms of |term|).  margin_e / margin_g: distance
  * (A) to the nearest energy discontinuity (grid boundary) / gradient kink
  * (cell face).                                                               */
 static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, const double X[3], double grad[3],
-                         double* abs_e, double abs_g[3], double* abs_h, double* margin_e, double* margin_g) {
+                         double* abs_e, double* margin_e, double* margin_g) {
     const int n[3] = {G->nx, G->ny, G->nz};
     const double h = G->spacing;
     double u[3];
@@ -168,10 +168,8 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
             const double c = 0.5 * (double)(n[k] - 1);
             E += F->w_out * (u[k] - c) * (u[k] - c);
             grad[k] = 2.0 * F->w_out * (u[k] - c) / h;
-            abs_g[k] = fabs(grad[k]);
         }
         *abs_e = fabs(E);
-        *abs_h = 2.0 * F->w_out / (h * h);
         return E;
     }
     int i0[3];
@@ -183,7 +181,7 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
     const int m_e = G->n_maps - 2, m_d = G->n_maps - 1;
     const double coef[3] = {1.0, q, fabs(q)};
     const int mm[3] = {map, m_e, m_d};
-    double E = 0.0, dEdu[3] = {0.0, 0.0, 0.0}, aE = 0.0, aG[3] = {0.0, 0.0, 0.0}, aV = 0.0;
+    double E = 0.0, dEdu[3] = {0.0, 0.0, 0.0}, aE = 0.0;
     for (int cz = 0; cz < 2; cz++)
         for (int cy = 0; cy < 2; cy++)
             for (int cx = 0; cx < 2; cx++) {
@@ -199,25 +197,17 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
                     const double v = coef[t] * gv(G, mm[t], i0[0] + cx, i0[1] + cy, i0[2] + cz);
                     E += wgt * v;
                     aE += fabs(wgt * v);
-                    aV += fabs(v);
-                    for (int k = 0; k < 3; k++) {
-                        dEdu[k] += dw[k] * v;
-                        aG[k] += fabs(dw[k] * v);
-                    }
+                    for (int k = 0; k < 3; k++) dEdu[k] += dw[k] * v;
                 }
             }
-    for (int k = 0; k < 3; k++) {
-        grad[k] = dEdu[k] / h;
-        abs_g[k] = aG[k] / h;
-    }
+    for (int k = 0; k < 3; k++) grad[k] = dEdu[k] / h;
     *abs_e = aE;
-    *abs_h = aV / (h * h);
     return E;
 }
 
 /* O-3: IntraGradient for one pair at distance r.
- * Returns E; *dEdr = dE/dr.  *abs_e = |cA s^-m| + |cB s^-n| + |E_el| + |E_ds|,
- * *abs_d = the same for dE/dr.  Smoothing (Z6): delta = smooth/2,
+ * Returns E; *dEdr = dE/dr.  *abs_e = |cA s^-m| + |cB s^-n| + |E_el| + |E_ds|
+ * (the Z18 magnitude sum).  Smoothing (Z6): delta = smooth/2,
  *   s = r + delta if r <= r0 - delta; s = r0 if r < r0 + delta; else r - delta.
  * vdW / H-bond if r < cut_vdw (Z7):  E = cA s^-m - cB s^-n  (Z10).
  * electrostatics if r < cut_el:      E = c_el qi qj / (r_e eps(r_e)),
@@ -225,12 +215,12 @@ static double inter_atom(const ado_grid* G, const ado_ff* F, int map, double q, 
  * desolvation if r < cut_el:
  *   E = c_ds [(S_i + Q|q_i|) V_j + (S_j + Q|q_j|) V_i] exp(-r^2 / (2 sigma^2)). */
 static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, double r, double* dEdr, double* abs_e,
-                         double* abs_d, double* abs_dd, double* margin_e, double* margin_g) {
+                         double* margin_e, double* margin_g) {
     const int ti = L->atom_type[i], tj = L->atom_type[j];
     const float* tp = L->tp_coef + ((size_t)ti * L->n_types + tj) * 5;
     const double cA = tp[0], cB = tp[1], r0 = tp[2], m = tp[3], nn = tp[4];
     const double qi = L->charge[i], qj = L->charge[j];
-    double E = 0.0, D = 0.0, aE = 0.0, aD = 0.0, aDD = 0.0;
+    double E = 0.0, D = 0.0, aE = 0.0;
     const double delta = 0.5 * F->smooth;
     double me = fmin(fabs(r - F->cut_vdw), fabs(r - F->cut_el));
     double mg = fmin(fmin(fabs(r - (r0 - delta)), fabs(r - (r0 + delta))), fabs(r - F->el_rmin));
@@ -244,8 +234,6 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         const double da = -m * cA * pow(s, -m - 1.0) * dsdr, db = -nn * cB * pow(s, -nn - 1.0) * dsdr;
         D += da - db;
         aE += fabs(ea) + fabs(eb);
-        aD += fabs(da) + fabs(db);
-        aDD += dsdr * (m * (m + 1.0) * fabs(cA) * pow(s, -m - 2.0) + nn * (nn + 1.0) * fabs(cB) * pow(s, -nn - 2.0));
     }
     if (r < F->cut_el) {
         const double lB = F->diel_lambda * F->diel_B;
@@ -259,8 +247,6 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         E += eel;
         D += del;
         aE += fabs(eel);
-        aD += fabs(del);
-        aDD += 2.0 * fabs(del) / re;
         const double Si = L->type_S[ti], Sj = L->type_S[tj], Vi = L->type_V[ti], Vj = L->type_V[tj];
         const double pref = F->coeff_ds * ((Si + F->qasp * fabs(qi)) * Vj + (Sj + F->qasp * fabs(qj)) * Vi);
         const double s2 = F->sigma_ds * F->sigma_ds;
@@ -269,13 +255,9 @@ static double intra_pair(const ado_ligand* L, const ado_ff* F, int i, int j, dou
         E += eds;
         D += dds;
         aE += fabs(eds);
-        aD += fabs(dds);
-        aDD += fabs(eds) * (r * r / (s2 * s2) + 1.0 / s2);
     }
     *dEdr = D;
     *abs_e = aE;
-    *abs_d = aD;
-    *abs_dd = aDD;
     *margin_e = me;
     *margin_g = mg;
     return E;
@@ -325,69 +307,65 @@ static void jacobian(const ado_ligand* L, const ado_grid* G, const double* g, co
 
 /* One pose: E (O-5: inter + intra), gene gradient grad[G] (may be NULL),
  * aux[AUX_N] (may be NULL), agrad[G] (may be NULL), X_out [N][3] (may be NULL).
- * Condition numbers for the Z18 tolerance:
- *   aux[AUX_ABS_E]  = sum over every energy term of |term|
- *   aux[AUX_SENS_E] = sum over terms of |d term / d coordinates| x |coordinates|
- *                     (first-order sensitivity of E to relative rounding of X)
- *   agrad[k]        = sum over terms of |dX/dg_k| . (|term gradient| +
- *                     |d term gradient / dX| x |X|)                         */
+ * Scales of the Z18 tolerance:
+ *   aux[AUX_ABS_E] = A_E = sum over every energy term of |term|
+ *   agrad[k]       = A_grad[k] = sum of |summand| over the summands of the O-4
+ *                    chain rule dE/dg_k = sum_i dX_i/dg_k . g_i, with g_i split
+ *                    into its terms: |dX_i/dg_k . g_inter,i| per atom and
+ *                    |dX_i/dg_k . F_p| + |dX_j/dg_k . F_p| per intra pair p
+ *                    (F_p = dE_p/dr d_hat, the pair's force on i and on j).
+ * aux[AUX_MARGIN_E] / aux[AUX_MARGIN_G]: distance (A) to the nearest energy
+ * discontinuity (grid boundary, cutoff) / gradient kink (cell face, smoothing
+ * band edge, electrostatic floor).
+ * aux[AUX_SENS_E] = S_E, used ONLY by the separately labelled clash gate
+ * (A_E >= 500): the first-order change of E when every
+ * atom coordinate moves by its own length, sum_i |grad E_inter,i|_2 |X_i|_2 +
+ * sum_p |dE_p/dr| (|X_i|_2 + |X_j|_2) -- times 2^-20 it bounds what rounding
+ * the coordinates to 16 FP32 ulps can do to E.                              */
 int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const double* g, double* E_out, double* grad,
              double* aux, double* agrad, double* X_out) {
     const int N = L->n_atoms, Gn = 6 + L->n_tors;
     double* X = (double*)malloc(sizeof(double) * 3 * N);
     double* gi = (double*)calloc((size_t)3 * N, sizeof(double)); /* atom gradients */
-    double* ag = (double*)calloc((size_t)3 * N, sizeof(double)); /* abs atom gradients (inter) */
     double* J = (double*)malloc(sizeof(double) * 3 * (size_t)N * Gn);
     double* acc = agrad ? (double*)calloc((size_t)Gn, sizeof(double)) : NULL;
-    if (!X || !gi || !ag || !J) return -4;
+    if (!X || !gi || !J || (agrad && !acc)) return -4;
     double T[3];
     ado_pose(L, G, g, X, T);
     jacobian(L, G, g, X, T, J);
     double Einter = 0.0, Eintra = 0.0, AE = 0.0, ME = 1e30, MG = 1e30, SE = 0.0;
-    /* |J| row norms per atom and gene (for the condition numbers) */
     for (int i = 0; i < N; i++) {
-        const double xn = sqrt(dot(X + 3 * i, X + 3 * i));
-        double gr[3], agr[3], ae, ah, me, mg;
-        Einter += inter_atom(G, F, L->atom_map[i], (double)L->charge[i], X + 3 * i, gr, &ae, agr, &ah, &me, &mg);
+        double gr[3], ae, me, mg;
+        Einter += inter_atom(G, F, L->atom_map[i], (double)L->charge[i], X + 3 * i, gr, &ae, &me, &mg);
         AE += ae;
-        SE += (agr[0] + agr[1] + agr[2]) * xn;      /* first-order sensitivity to coordinate rounding */
+        SE += sqrt(dot(gr, gr)) * sqrt(dot(X + 3 * i, X + 3 * i));
         ME = fmin(ME, me);
         MG = fmin(MG, mg);
-        for (int k = 0; k < 3; k++) { gi[3 * i + k] += gr[k]; ag[3 * i + k] += agr[k]; }
+        for (int k = 0; k < 3; k++) gi[3 * i + k] += gr[k];
         if (acc)
-            for (int q = 0; q < Gn; q++) {
-                const double* Jq = J + ((size_t)i * Gn + q) * 3;
-                const double jn = fabs(Jq[0]) + fabs(Jq[1]) + fabs(Jq[2]);
-                acc[q] += fabs(Jq[0]) * agr[0] + fabs(Jq[1]) * agr[1] + fabs(Jq[2]) * agr[2] + jn * ah * xn;
-            }
+            for (int q = 0; q < Gn; q++) acc[q] += fabs(dot(J + ((size_t)i * Gn + q) * 3, gr));
     }
     for (int p = 0; p < L->n_pairs; p++) {
         const int i = L->pairs[2 * p], j = L->pairs[2 * p + 1];
         double d[3];
         for (int k = 0; k < 3; k++) d[k] = X[3 * i + k] - X[3 * j + k];
         const double r = sqrt(dot(d, d));
-        double dEdr, ae, ad, add, me, mg;
-        Eintra += intra_pair(L, F, i, j, r, &dEdr, &ae, &ad, &add, &me, &mg);
-        const double xl = sqrt(dot(X + 3 * i, X + 3 * i)) + sqrt(dot(X + 3 * j, X + 3 * j));
+        double dEdr, ae, me, mg;
+        Eintra += intra_pair(L, F, i, j, r, &dEdr, &ae, &me, &mg);
         AE += ae;
-        SE += ad * xl;
+        SE += fabs(dEdr) * (sqrt(dot(X + 3 * i, X + 3 * i)) + sqrt(dot(X + 3 * j, X + 3 * j)));
         ME = fmin(ME, me);
         MG = fmin(MG, mg);
         if (r > 0.0) {
+            double fp[3];
             for (int k = 0; k < 3; k++) {
-                const double fk = dEdr * d[k] / r;
-                gi[3 * i + k] += fk;
-                gi[3 * j + k] -= fk;
+                fp[k] = dEdr * d[k] / r;
+                gi[3 * i + k] += fp[k];
+                gi[3 * j + k] -= fp[k];
             }
-            if (acc) {
-                const double fa[3] = {fabs(ad * d[0] / r), fabs(ad * d[1] / r), fabs(ad * d[2] / r)};
-                const double h2 = (add + ad / r) * xl;   /* |dF/dX| x coordinate magnitude */
-                for (int q = 0; q < Gn; q++) {
-                    const double* Ji = J + ((size_t)i * Gn + q) * 3;
-                    const double* Jj = J + ((size_t)j * Gn + q) * 3;
-                    for (int k = 0; k < 3; k++) acc[q] += (fabs(Ji[k]) + fabs(Jj[k])) * (fa[k] + h2);
-                }
-            }
+            if (acc)
+                for (int q = 0; q < Gn; q++)
+                    acc[q] += fabs(dot(J + ((size_t)i * Gn + q) * 3, fp)) + fabs(dot(J + ((size_t)j * Gn + q) * 3, fp));
         }
     }
     if (grad)
@@ -413,7 +391,6 @@ int ado_eval(const ado_ligand* L, const ado_grid* G, const ado_ff* F, const doub
     if (X_out) memcpy(X_out, X, sizeof(double) * 3 * N);
     free(X);
     free(gi);
-    free(ag);
     free(J);
     free(acc);
     return 0;
@@ -458,10 +435,14 @@ int ado_adadelta_step(int32_t n_genes, const double* grad, double* eg2, double* 
  * (300 by default).  Each iteration: (E, grad) = eval(genes); keep the
  * genotype if E < best_E (strict, earliest wins, Z15); update all genes.  The
  * update after the last eval is not evaluated (Z15).  No angle wrapping (Z16).
- * Outputs: best_genes [n][stride] (double), best_E [n]. */
+ * Outputs: best_genes [n][stride] (double), best_E [n], and (trace != NULL)
+ * for every step (E, A_E, S_E, margin_e, margin_g) of the evaluated genotype,
+ * trace [n][max_iters][5] (Z19 ii free-running trajectories: the gate scales
+ * of the step and its distances to the nearest energy discontinuity / gradient
+ * kink). */
 int ado_local_search(const ado_ligand* L, const ado_grid* G, const ado_ff* F, int32_t n_poses, const float* genes,
                      int32_t stride, int32_t max_iters, double rho, double eps, double* best_genes, double* best_E,
-                     int32_t n_threads) {
+                     double* trace, int32_t n_threads) {
     const int Gn = 6 + L->n_tors;
     if (stride < Gn) return -1;
     int err = 0;
@@ -478,9 +459,17 @@ int ado_local_search(const ado_ligand* L, const ado_grid* G, const ado_ff* F, in
         }
         double bE = INFINITY;
         for (int it = 0; it < max_iters; it++) {
-            double E;
-            int rc = ado_eval(L, G, F, x, &E, gr, NULL, NULL, NULL);
+            double E, aux[AUX_N];
+            int rc = ado_eval(L, G, F, x, &E, gr, trace ? aux : NULL, NULL, NULL);
             if (rc) err = rc;
+            if (trace) {
+                double* t = trace + ((size_t)p * max_iters + it) * 5;
+                t[0] = E;
+                t[1] = aux[AUX_ABS_E];
+                t[2] = aux[AUX_SENS_E];
+                t[3] = aux[AUX_MARGIN_E];
+                t[4] = aux[AUX_MARGIN_G];
+            }
             if (E < bE) {
                 bE = E;
                 for (int q = 0; q < Gn; q++) best[q] = x[q];

@@ -60,7 +60,7 @@ def lib():
             L.ado_score.argtypes = [P, P, P, C.c_int32, P, C.c_int32, P, P, P, P, C.c_int32]
             L.ado_adadelta_step.argtypes = [C.c_int32, P, P, P, P, C.c_double, C.c_double]
             L.ado_local_search.argtypes = [P, P, P, C.c_int32, P, C.c_int32, C.c_int32, C.c_double, C.c_double,
-                                           P, P, C.c_int32]
+                                           P, P, P, C.c_int32]
             L.ado_best_of_run.argtypes = [C.c_int32, C.c_int32, P, P]
             L.ado_exact_sum.argtypes = [P, C.c_int64, C.c_int64]
             L.ado_exact_sum.restype = C.c_double
@@ -142,16 +142,20 @@ def score(lig, grid, ff, genes: np.ndarray, threads: int = 0):
     return E, gr, aux, ag
 
 
-def local_search(lig, grid, ff, genes: np.ndarray, max_iters=300, rho=0.8, eps=0.01, threads: int = 0):
+def local_search(lig, grid, ff, genes: np.ndarray, max_iters=300, rho=0.8, eps=0.01, threads: int = 0,
+                 trace: bool = False):
+    """O-6 from FP32 start genotypes [n, stride]: (best_genes, best_E) and, with
+    trace=True, (E, A_E, S_E, margin_e, margin_g) of every step [n, max_iters, 5] as a third output."""
     lg, g, f, keep = _structs(lig, grid, ff)
     genes = np.ascontiguousarray(genes, dtype=np.float32)
     n, stride = genes.shape
     best = np.zeros((n, stride))
     bE = np.zeros(n)
+    tE = np.zeros((n, max_iters, 5)) if trace else None
     rc = lib().ado_local_search(C.byref(lg), C.byref(g), C.byref(f), n, _ptr(genes), stride, max_iters, rho, eps,
-                                _ptr(best), _ptr(bE), threads or os.cpu_count())
+                                _ptr(best), _ptr(bE), _ptr(tE) if trace else None, threads or os.cpu_count())
     assert rc == 0, rc
-    return best, bE
+    return (best, bE, tE) if trace else (best, bE)
 
 
 def adadelta_step(grad, eg2, ed2, genes, rho=0.8, eps=0.01):
