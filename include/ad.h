@@ -17,7 +17,9 @@
  *     stream).  Compute calls enqueue asynchronously and return; a kernel fault
  *     surfaces as AD_ERR_CUDA on a later call or stream synchronisation.
  *     Device-side argument errors (bad pose_ligand ids) surface as
- *     AD_ERR_INVALID_ARG on the NEXT call on the same context.
+ *     AD_ERR_INVALID_ARG on a later call on the same context once the
+ *     offending kernel has completed (no call blocks to find out), or at
+ *     ad_sync().
  *   - One context per device per host thread, except ad_upload_ligand and
  *     ad_free_ligand, which may be called concurrently from several host threads
  *     on one context (the host-side ligand preparation -- torsion tree, pair
@@ -303,6 +305,15 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
  * n_partials in {32, 64, ..., 1024} (multiple of 32), n_comp in 1..64. */
 int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
                          const float* partials, float* out, void* cuda_stream);
+
+/* Wait for `cuda_stream` and report any device-side argument error recorded by
+ * kernels enqueued so far (bad pose_ligand ids, a ligand outside the launch
+ * set's footprint, CTA groups mixing ligands, a ligand with more genes than
+ * geno_stride): AD_ERR_INVALID_ARG with the reasons in ad_last_error(), then
+ * the error word is cleared.  Compute calls never block for this: they report
+ * an error word once the work that set it has completed.  AD_ERR_CUDA for a
+ * kernel fault. */
+int32_t ad_sync(ad_context* ctx, void* cuda_stream);
 
 /* Device properties useful to callers: number of SMs and the shared memory
  * footprint (bytes) the SIMT/TC kernel uses per pose for ligand `lig`. */

@@ -24,7 +24,8 @@ ENGINES = {"simt": AD_ENGINE_SIMT, "tc": AD_ENGINE_TC, "paper": AD_ENGINE_PAPER_
 # names exported by include/ad.h (tests check the .so exports all of them)
 EXPORTS = ("ad_last_error", "ad_version", "ad_context_create", "ad_context_destroy", "ad_upload_grids",
            "ad_upload_ligand", "ad_free_ligand", "ad_set_launch_ligands", "ad_set_schedule_effort",
-           "ad_score_poses", "ad_local_search", "ad_lga_run", "ad_reduce_blocks", "ad_query", "ad_last_launch")
+           "ad_score_poses", "ad_local_search", "ad_lga_run", "ad_reduce_blocks", "ad_sync", "ad_query",
+           "ad_last_launch")
 
 
 class AdError(RuntimeError):
@@ -89,6 +90,7 @@ def lib():
             L.ad_local_search.argtypes = [P, I32, P, I32, P, I32, P, P, P, C.POINTER(LSParams), P]
             L.ad_reduce_blocks.argtypes = [P, I32, I32, I32, I32, P, P, P]
             L.ad_lga_run.argtypes = [P, I32, I32, P, I32, P, P, P, P, C.POINTER(LGAParams), P]
+            L.ad_sync.argtypes = [P, P]
             L.ad_query.argtypes = [P, I32, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
             L.ad_last_launch.argtypes = [P, C.POINTER(I32), C.POINTER(I32), C.POINTER(I32)]
             for name in EXPORTS:
@@ -220,6 +222,11 @@ def ad_reduce_blocks(ctx, engine, partials, out, stream=None) -> None:
                                   _stream(stream)))
 
 
+def ad_sync(ctx, stream=None) -> None:
+    """Wait for the stream; raise AdError for device-side argument errors recorded so far."""
+    _check(lib().ad_sync(ctx, _stream(stream)))
+
+
 def ad_query(ctx, lig=-1):
     a, b, c = C.c_int32(), C.c_int32(), C.c_int32()
     _check(lib().ad_query(ctx, lig, C.byref(a), C.byref(b), C.byref(c)))
@@ -277,6 +284,10 @@ class Context:
         n = threads or max(1, min(len(ligs), len(os.sched_getaffinity(0))))
         with ThreadPoolExecutor(n) as ex:
             return list(ex.map(lambda L: ad_upload_ligand(self.h, L, ff), ligs))
+
+    def sync(self) -> None:
+        """ad_sync on the current stream: raises AdError for device-side errors."""
+        ad_sync(self.h)
 
     def free_ligand(self, lig_id: int) -> None:
         ad_free_ligand(self.h, lig_id)

@@ -83,6 +83,17 @@ struct ad_context {
     LigDev* d_ligtab = nullptr;
     int32_t ligtab_cap = 0;
     int32_t* d_err = nullptr;
+    // device error word read back asynchronously: after every launch a 4-byte copy
+    // d_err -> h_err (pinned) and an event on the caller's stream; later calls
+    // report it once the event has completed (no host-device synchronisation)
+    int32_t* h_err = nullptr;
+    cudaEvent_t err_ev = nullptr;
+    bool err_pending = false;
+    // launch-shape caches: cudaFuncSetAttribute once per kernel, occupancy per
+    // (kernel, threads, dynamic shared memory)
+    std::mutex launch_mu;
+    std::vector<const void*> smem_opted;
+    std::vector<std::array<long long, 4>> occ;  // {kernel, threads, smem, blocks}
     // AD_INTRA_MODE=owner|scatter at context creation (tuning knob; scatter measured
     // faster on config 2: 1.40e8 vs 1.26e8 evals/s, profiles/README.md)
     int intra_mode = INTRA_SCATTER;
@@ -107,17 +118,63 @@ int32_t set_device(ad_context* ctx) {
     return AD_OK;
 }
 
-// surfaces device-side argument errors recorded by earlier kernels
-int32_t check_device_err(ad_context* ctx) {
-    int32_t h = 0;
-    CUDA_TRY(cudaMemcpy(&h, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost));
+int32_t report_device_err(int32_t h) {
+    return fail(AD_ERR_INVALID_ARG, "a previous kernel reported %s%s%s%s",
+                (h & ERR_BAD_LIGAND) ? "[pose_ligand id out of range] " : "",
+                (h & ERR_FOOTPRINT) ? "[ligand footprint larger than the launch's] " : "",
+                (h & ERR_MIXED_CTA) ? "[pose_ligand not uniform within a CTA group] " : "",
+                (h & ERR_STRIDE) ? "[geno_stride < 6 + n_tors of a pose's ligand]" : "");
+}
+
+// Surfaces device-side argument errors recorded by earlier kernels without
+// blocking: the error word of the last completed read-back (see read_back_err).
+// The word is sticky on the device until reported, then cleared in stream order.
+int32_t check_device_err(ad_context* ctx, cudaStream_t st) {
+    if (!ctx->err_pending) return AD_OK;
+    const cudaError_t q = cudaEventQuery(ctx->err_ev);
+    if (q == cudaErrorNotReady) return AD_OK;
+    if (q != cudaSuccess) return fail(AD_ERR_CUDA, "error read-back: %s", cudaGetErrorString(q));
+    ctx->err_pending = false;
+    const int32_t h = *ctx->h_err;
     if (h) {
-        CUDA_TRY(cudaMemset(ctx->d_err, 0, sizeof(int32_t)));
-        return fail(AD_ERR_INVALID_ARG, "a previous kernel reported %s%s%s",
-                    (h & ERR_BAD_LIGAND) ? "[pose_ligand id out of range] " : "",
-                    (h & ERR_FOOTPRINT) ? "[ligand footprint larger than `lig`'s] " : "",
-                    (h & ERR_MIXED_CTA) ? "[pose_ligand not uniform within a CTA group]" : "");
+        *ctx->h_err = 0;
+        CUDA_TRY(cudaMemsetAsync(ctx->d_err, 0, sizeof(int32_t), st));
+        return report_device_err(h);
     }
+    return AD_OK;
+}
+
+// Enqueue the read-back of the device error word after this call's launches.
+int32_t read_back_err(ad_context* ctx, cudaStream_t st) {
+    CUDA_TRY(cudaMemcpyAsync(ctx->h_err, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaEventRecord(ctx->err_ev, st));
+    ctx->err_pending = true;
+    return AD_OK;
+}
+
+// Raise a kernel's dynamic shared-memory limit to the device maximum, once.
+int32_t opt_in_smem(ad_context* ctx, const void* k) {
+    std::lock_guard<std::mutex> lock(ctx->launch_mu);
+    if (std::find(ctx->smem_opted.begin(), ctx->smem_opted.end(), k) != ctx->smem_opted.end()) return AD_OK;
+    CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin));
+    ctx->smem_opted.push_back(k);
+    return AD_OK;
+}
+
+// Resident CTAs per SM of kernel k at (threads, smem), cached.
+int32_t occupancy(ad_context* ctx, const void* k, int threads, size_t smem, int* blocks) {
+    {
+        std::lock_guard<std::mutex> lock(ctx->launch_mu);
+        for (const auto& e : ctx->occ)
+            if (e[0] == (long long)(uintptr_t)k && e[1] == threads && e[2] == (long long)smem) {
+                *blocks = (int)e[3];
+                return AD_OK;
+            }
+    }
+    if (int32_t rc = opt_in_smem(ctx, k)) return rc;
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, k, threads, smem));
+    std::lock_guard<std::mutex> lock(ctx->launch_mu);
+    ctx->occ.push_back({(long long)(uintptr_t)k, threads, (long long)smem, *blocks});
     return AD_OK;
 }
 
@@ -974,12 +1031,16 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
 // Records of a cherry schedule (layout: ad_internal.h pka / pkb / pkc, kernel:
 // intra_cherry).  Empty ends and lanes get a zero-charge X row and a spare
 // gradient row in the bank group least used by that access in their
-// quarter-warp (distinct groups within a lane).
+// quarter-warp (distinct groups within a lane).  Row indices are 8-bit: X row
+// (< npad + 8) and gradient row k * npad + row (< K * npad + 8), both <= 255
+// (cherry_rows_fit).
 struct CherryRecords {
     std::vector<uint4> a;
     std::vector<float4> b, c;
 };
-CherryRecords pack_cherries(const CherrySchedule& S, int npad, int ws_g, const std::vector<int>& ptp,
+bool cherry_rows_fit(int npad, int K) { return npad + 8 <= 256 && K * npad + 8 <= 256; }
+
+CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector<int>& ptp,
                             const std::vector<float4>& tp, const std::vector<float>& pdsv) {
     CherryRecords R;
     const size_t n = (size_t)S.steps * 32;
@@ -987,8 +1048,6 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, int ws_g, const s
     R.b.resize(n);
     R.c.resize(n);
     const int K = S.slots;
-    auto xoff = [&](int row) { return (uint32_t)(16 * row); };
-    auto goff = [&](int row, int k) { return (uint32_t)(ws_g + 16 * (k * npad + row)); };
     for (size_t q0 = 0; q0 < n; q0 += 8) {  // one quarter-warp
         int cnt[3][8] = {};
         for (size_t q = q0; q < q0 + 8; ++q) {
@@ -1000,7 +1059,7 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, int ws_g, const s
         }
         for (size_t q = q0; q < q0 + 8; ++q) {
             const CherryLane& L = S.lane[q];
-            uint32_t w[3];
+            uint32_t xr[3], gr[3];
             unsigned taken = 0;  // bank groups of this lane's dummy rows (distinct positions)
             auto dummy = [&](int acc) {
                 int r = -1;
@@ -1008,28 +1067,40 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, int ws_g, const s
                     if (!(taken >> x & 1u) && (r < 0 || cnt[acc][x] < cnt[acc][r])) r = x;
                 taken |= 1u << r;
                 cnt[acc][r]++;
-                return xoff(npad + r) | (goff(r, K) << 16);
+                xr[acc] = (uint32_t)(npad + r);
+                gr[acc] = (uint32_t)(K * npad + r);
             };
-            w[0] = L.c >= 0 ? xoff(L.c) | (goff(L.c, L.kc) << 16) : dummy(0);
-            float4 co[2];
-            float dsv[2];
+            if (L.c >= 0) {
+                xr[0] = (uint32_t)L.c;
+                gr[0] = (uint32_t)(L.kc * npad + L.c);
+            } else {
+                dummy(0);
+            }
+            float cA[2], cB[2], cC[2], r0[2], dsv[2];
             for (int k = 0; k < 2; ++k) {
                 if (L.c >= 0 && L.e[k] >= 0) {
-                    w[1 + k] = xoff(L.e[k]) | (goff(L.e[k], L.ke[k]) << 16);
-                    const float4 t = tp[ptp[L.p[k]]];
-                    co[k] = make_float4(t.x, t.y, t.w > 8.f ? -t.z : t.z, 0.f);  // sign bit: 12-10 pair
+                    xr[1 + k] = (uint32_t)L.e[k];
+                    gr[1 + k] = (uint32_t)(L.ke[k] * npad + L.e[k]);
+                    const float4 t = tp[ptp[L.p[k]]];  // (cA, cB, r0, n)
+                    const bool hb = t.w > 8.f;        // 12-10 pair: its s^-10 coefficient goes to cC
+                    cA[k] = t.x;
+                    cB[k] = hb ? 0.f : t.y;
+                    cC[k] = hb ? t.y : 0.f;
+                    r0[k] = t.z;
                     dsv[k] = pdsv[L.p[k]];
                 } else {
-                    w[1 + k] = dummy(1 + k);
-                    co[k] = make_float4(0.f, 0.f, 1.f, 0.f);
+                    dummy(1 + k);
+                    cA[k] = cB[k] = cC[k] = 0.f;
+                    r0[k] = 1.f;
                     dsv[k] = 0.f;
                 }
             }
-            uint32_t ud;
-            memcpy(&ud, &dsv[0], 4);
-            R.a[q] = make_uint4(w[0], w[1], w[2], ud);
-            R.b[q] = make_float4(co[0].x, co[0].y, co[0].z, dsv[1]);
-            R.c[q] = make_float4(co[1].x, co[1].y, co[1].z, 0.f);
+            uint32_t d0, d1;
+            memcpy(&d0, &dsv[0], 4);
+            memcpy(&d1, &dsv[1], 4);
+            R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16), gr[0] | (gr[1] << 8) | (gr[2] << 16), d0, d1);
+            R.b[q] = make_float4(cA[0], cA[1], cB[0], cB[1]);
+            R.c[q] = make_float4(r0[0], r0[1], cC[0], cC[1]);
         }
     }
     return R;
@@ -1247,6 +1318,9 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
         e = cudaDeviceGetAttribute(&ctx->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, cuda_device);
     if (e == cudaSuccess) e = cudaMalloc(&ctx->d_err, sizeof(int32_t));
     if (e == cudaSuccess) e = cudaMemset(ctx->d_err, 0, sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaHostAlloc(reinterpret_cast<void**>(&ctx->h_err), sizeof(int32_t), cudaHostAllocDefault);
+    if (e == cudaSuccess) *ctx->h_err = 0;
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->err_ev, cudaEventDisableTiming);
     if (e != cudaSuccess) {
         delete ctx;
         return fail(AD_ERR_CUDA, "context init: %s", cudaGetErrorString(e));
@@ -1267,6 +1341,8 @@ int32_t ad_context_destroy(ad_context* ctx) {
     if (ctx->d_ed) cudaFree(ctx->d_ed);
     if (ctx->d_ligtab) cudaFree(ctx->d_ligtab);
     if (ctx->d_err) cudaFree(ctx->d_err);
+    if (ctx->h_err) cudaFreeHost(ctx->h_err);
+    if (ctx->err_ev) cudaEventDestroy(ctx->err_ev);
     delete ctx;
     return AD_OK;
 }
@@ -1509,8 +1585,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         if (ctx->pk_smem_max > 0 && P > 0) {
             const int max_steps = std::min(ctx->pairs_smem_max / (kPairsPerStep * 12), ctx->pk_smem_max / (kLanes * 48));
             cs = schedule_cherries(npad_of(N), si, sj, ctx->sched_effort, max_steps);
-            const WarpScratch w = warp_scratch_layout(N, T, cs.slots, 0);
-            cherry = cs.steps <= max_steps && w.g + 16 * (npad_of(N) * (cs.slots + 1)) <= 0xffff;
+            cherry = cs.steps <= max_steps && cherry_rows_fit(npad_of(N), cs.slots);
         }
         // the prec list (the paper-style baseline's pairs; the warp engine's schedule
         // when it runs no cherries) is the pair-step schedule either way, so the
@@ -1539,6 +1614,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         mask[k] = make_uint2((uint32_t)m, (uint32_t)(m >> 32));
     }
     std::vector<float4> tors(2 * std::max(T, 1));
+    std::vector<double> tors64(6 * std::max(T, 1));
     std::vector<int4> tinfo(std::max(T, 1));
     for (int b = 0; b < T; ++b) {
         const int a0 = d->tors_axis[2 * b], c0 = d->tors_axis[2 * b + 1];
@@ -1548,6 +1624,10 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         if (!(nu > 0)) return fail(AD_ERR_INVALID_ARG, "torsion %d has a zero-length axis", b);
         tors[2 * b] = make_float4((float)P0[0], (float)P0[1], (float)P0[2], 0.f);
         tors[2 * b + 1] = make_float4((float)(u[0] / nu), (float)(u[1] / nu), (float)(u[2] / nu), 0.f);
+        for (int k = 0; k < 3; ++k) {
+            tors64[6 * b + k] = P0[k];
+            tors64[6 * b + 3 + k] = u[k] / nu;
+        }
         tinfo[b] = make_int4(slot[newi[a0]], slot[newi[c0]], lo[b], hi[b]);
     }
 
@@ -1605,6 +1685,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         h.off_atoms = B.put(atoms.data(), sizeof(float4) * N);
         h.off_info = B.put(info.data(), sizeof(int2) * N);
         h.off_tors = B.put(tors.data(), sizeof(float4) * 2 * T);
+        h.off_tors64 = B.put(tors64.data(), sizeof(double) * 6 * T);
         h.off_tinfo = B.put(tinfo.data(), sizeof(int4) * T);
         h.off_chain = B.put(chain.data(), chain.size());
         h.off_mask = B.put(mask.data(), sizeof(uint2) * N);
@@ -1613,7 +1694,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         o.ws = warp_scratch_layout(N, T, h.n_slots, own.C);
         if (warp_cherry) {
             // cherry records (ad_internal.h pka / pkb / pkc), staged with the tables
-            const CherryRecords cr = pack_cherries(cs, h.n_pad, o.ws.g, ptp, tp, pd);
+            const CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd);
             h.off_tp = h.off_prec = h.off_pdsv = h.off_pkg = 0;
             h.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
             B.put(cr.b.data(), sizeof(float4) * cr.b.size());
@@ -1667,7 +1748,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             h.stage_bytes = h.pairs_gmem ? h.off_prec : h.blob_bytes;
         }
         h.scratch_bytes = o.ws.bytes;
-        h.ws_g = o.ws.g; h.ws_w = o.ws.w; h.ws_d = o.ws.d; h.ws_trig = o.ws.trig;
+        h.ws_g = o.ws.g; h.ws_w = o.ws.w; h.ws_d = o.ws.d; h.ws_trig = o.ws.trig; h.ws_trig64 = o.ws.trig64;
         h.ws_tw = o.ws.tw; h.ws_genes = o.ws.genes; h.ws_part = o.ws.part;
         memcpy(B.buf.data(), &h, sizeof(h));
         o.buf = std::move(B.buf);
@@ -1816,6 +1897,16 @@ int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const 
     return AD_OK;
 }
 
+// pose_ligand launches: every ligand the launch may reference must fit the stride
+// (the kernels also check each pose's ligand on the device: ERR_STRIDE)
+int32_t check_launch_stride(ad_context* ctx, int32_t stride) {
+    int tmax = 0;
+    for_each_launch_ligand(ctx, [&](const LigSlot& o) { tmax = std::max(tmax, o.n_tors); });
+    if (stride < 6 + tmax)
+        return fail(AD_ERR_INVALID_ARG, "geno_stride %d < 6 + n_tors = %d of a ligand in the launch set", stride, 6 + tmax);
+    return AD_OK;
+}
+
 // pose_ligand launches may touch any live ligand; the scoring constants are kernel
 // parameters, so they must be identical across the live ligands
 int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
@@ -1866,9 +1957,8 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             if (p.pose_ligand && ((w & (w - 1)) || w > 8)) continue;  // ad.h: ligand runs are multiples of 8
             const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
             if (smem > (size_t)ctx->max_smem_optin) continue;
-            CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             int blocks = 0;
-            CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, k, w * 32, smem));
+            if (int32_t rc = occupancy(ctx, reinterpret_cast<const void*>(k), w * 32, smem, &blocks)) return rc;
             if (blocks <= 0) continue;
             const int active = blocks * w;
             const long ctas = (p.n_poses + w - 1) / w;
@@ -1930,9 +2020,11 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
     if (n_poses > 0 && !energy) return fail(AD_ERR_INVALID_ARG, "energy is NULL");
     if (pose_ligand) {
         if (int32_t rc = check_common_ff(ctx, lig)) return rc;
+        if (int32_t rc = check_launch_stride(ctx, geno_stride)) return rc;
     }
     if (int32_t rc = set_device(ctx)) return rc;
-    if (int32_t rc = check_device_err(ctx)) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (int32_t rc = check_device_err(ctx, st)) return rc;
     if (n_poses == 0) return AD_OK;
     KParams p = base_params(ctx, lig, pose_ligand, n_poses, geno_stride);
     p.genes = const_cast<float*>(genes);
@@ -1940,8 +2032,11 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
     p.grad = grad;
     p.aux = aux;
     const bool want_grad = grad != nullptr || aux != nullptr;
-    return launch_warp(ctx, ctx->ligs[lig], pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false, launch_is_wide(ctx, lig, pose_ligand)), p, 0,
-                       (cudaStream_t)stream, false);
+    if (int32_t rc = launch_warp(ctx, ctx->ligs[lig],
+                                 pick_warp_kernel(AD_ENGINE_SIMT, want_grad, false, launch_is_wide(ctx, lig, pose_ligand)),
+                                 p, 0, st, false))
+        return rc;
+    return read_back_err(ctx, st);
 }
 
 int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses, float* genes,
@@ -1955,13 +2050,14 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     if (n_poses > 0 && !best_energy) return fail(AD_ERR_INVALID_ARG, "best_energy is NULL");
     if (pose_ligand) {
         if (int32_t rc = check_common_ff(ctx, lig)) return rc;
+        if (int32_t rc = check_launch_stride(ctx, geno_stride)) return rc;
     }
     if (run_best && (prm->pop_per_run <= 0 || n_poses % prm->pop_per_run))
         return fail(AD_ERR_INVALID_ARG, "run_best needs pop_per_run > 0 dividing n_poses");
     if (int32_t rc = set_device(ctx)) return rc;
-    if (int32_t rc = check_device_err(ctx)) return rc;
-    if (n_poses == 0) return AD_OK;
     cudaStream_t st = (cudaStream_t)stream;
+    if (int32_t rc = check_device_err(ctx, st)) return rc;
+    if (n_poses == 0) return AD_OK;
     KParams p = base_params(ctx, lig, pose_ligand, n_poses, geno_stride);
     p.genes = genes;
     p.energy = best_energy;
@@ -1989,7 +2085,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         if (smem > (size_t)ctx->max_smem_optin) return fail(AD_ERR_LIMIT, "ligand too large for the baseline engine");
         void (*kern)(const KParams) = p.phase_cycles ? (tcec ? k_block_baseline<true, true> : k_block_baseline<false, true>)
                                                      : (tcec ? k_block_baseline<true> : k_block_baseline<false>);
-        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        if (int32_t rc = opt_in_smem(ctx, reinterpret_cast<const void*>(kern))) return rc;
         p.smem_blob = blob;
         p.smem_scratch = bscr;
         kern<<<n_poses, threads, smem, st>>>(p);
@@ -2015,7 +2111,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
                                                       runs, run_best);
         CUDA_TRY(cudaGetLastError());
     }
-    return AD_OK;
+    return read_back_err(ctx, st);
 }
 
 int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* genes, int32_t geno_stride,
@@ -2038,9 +2134,9 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
     if (prm->elitism < 0 || prm->elitism > pop || prm->max_gens < 0 || prm->max_evals < 0)
         return fail(AD_ERR_INVALID_ARG, "bad GA parameters");
     if (int32_t rc = set_device(ctx)) return rc;
-    if (int32_t rc = check_device_err(ctx)) return rc;
-    if (n_ind == 0) return AD_OK;
     cudaStream_t st = (cudaStream_t)stream;
+    if (int32_t rc = check_device_err(ctx, st)) return rc;
+    if (n_ind == 0) return AD_OK;
     const LigSlot& L = ctx->ligs[lig];
     const int S = geno_stride;
     GaParams G{pop, 6 + L.n_tors, S, prm->elitism, prm->cross_rate, prm->mut_rate, prm->tour_rate, prm->ls_rate,
@@ -2144,7 +2240,7 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
     LGA_TRY(cudaStreamSynchronize(st));
 #undef LGA_TRY
     cleanup();
-    return AD_OK;
+    return read_back_err(ctx, st);
 }
 
 int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
@@ -2260,6 +2356,22 @@ int32_t ad_last_launch(ad_context* ctx, int32_t* grid, int32_t* block, int32_t* 
     if (grid) *grid = ctx->last_grid;
     if (block) *block = ctx->last_block;
     if (smem_bytes) *smem_bytes = ctx->last_smem;
+    return AD_OK;
+}
+
+int32_t ad_sync(ad_context* ctx, void* stream) {
+    if (!ctx) return fail(AD_ERR_INVALID_ARG, "ctx is NULL");
+    if (int32_t rc = set_device(ctx)) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    CUDA_TRY(cudaStreamSynchronize(st));
+    int32_t h = 0;
+    CUDA_TRY(cudaMemcpy(&h, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    ctx->err_pending = false;
+    *ctx->h_err = 0;
+    if (h) {
+        CUDA_TRY(cudaMemset(ctx->d_err, 0, sizeof(int32_t)));
+        return report_device_err(h);
+    }
     return AD_OK;
 }
 

@@ -9,6 +9,7 @@
 //   info    int2   [N]      {map | type<<8 | chain_len<<16 | slot<<24, chain_start}; slot =
 //                           the atom's storage row in the per-pose X / gradient arrays
 //   tors    float4 [T][2]   reference-frame axis point P_b and unit axis u_b
+//   tors64  double [T][6]   the same in FP64 (u_b normalised in FP64), for the torsion chain
 //   tinfo   int4   [T]      {a_b, c_b, lo_b, hi_b}: axis atoms (storage rows) and the moving set
 //                           M_b = [lo_b, hi_b) (contiguous thanks to DFS order)
 //   chain   u8     [Lrot]   per atom: the torsions moving it, leaf -> root
@@ -86,7 +87,9 @@ struct alignas(16) LigHeader {
                                                         //      off_pk: cherry records (0 = none); base_*: steps
                                                         //      and slots of the prec list (= n_rounds / n_slots
                                                         //      unless the warp engine runs a cherry schedule)
-    int32_t off_pkg, reserved1, reserved2, reserved3;   // 160  off_pkg: pre-decoded global-memory places (0 = none)
+    int32_t off_pkg, off_tors64, ws_trig64, reserved3;  // 160  off_pkg: pre-decoded global-memory places (0 = none);
+                                                        //      off_tors64: double [T][6] axis point P_b, unit axis u_b
+                                                        //      (the FP64 torsion chain); ws_trig64: per-warp double2 [T]
     float ff[FF_N];                                     // 224
 };
 static_assert(sizeof(LigHeader) == 224, "header size");
@@ -125,7 +128,8 @@ struct WarpScratch {
     int32_t g;      // float4 [K][Npad]+8   atom gradient accumulators (slot 0 seeded with inter) + 8 spare
     int32_t w;      // float4 [Npad+1][2]   W staging (TC engines only)
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
-    int32_t trig;   // float2 [T]           cos, sin of torsion angles
+    int32_t trig;   // float2 [T+3]         cos, sin of torsion angles, then phi, theta, alpha/2
+    int32_t trig64; // double2 [T]          sin, 1 - cos of torsion angles in FP64 (the chain)
     int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
     int32_t genes;  // float  [64]
     int32_t part;   // float4 [C][32]       owner mode: per-(lane, chunk) partial gradients
@@ -148,6 +152,7 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     // row K: empty schedule places only ever target K * npad + (0..7)
     s.g = o;     o += 16 * npad * n_slots + 16 * 8;
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
+    s.trig64 = o; o += 16 * n_tors;
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
     s.genes = o; o += 4 * kMaxGenes;
     s.part = o;  o += 16 * 32 * n_chunks;
@@ -164,7 +169,7 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
 
 // Baseline engine (one block per pose) shared-memory layout after the blob.
 struct BlockScratch {
-    int32_t x, g, trig, tw, tacc, red, genes, stage, bytes;
+    int32_t x, g, trig, trig64, tw, tacc, red, genes, stage, bytes;
 };
 
 // stage: [stage_threads][8] floats for the TCEC variant's tensor-core reduction
@@ -177,6 +182,7 @@ __host__ __device__ inline BlockScratch block_scratch_layout(int32_t n_atoms, in
     s.x = o;     o += 16 * npad;
     s.g = o;     o += 16 * npad;
     s.trig = o;  o += align16(8 * (n_tors + 3));
+    s.trig64 = o; o += 16 * t1;
     s.tw = o;    o += 32 * t1;
     s.tacc = o;  o += align16(4 * t1);
     s.red = o;   o += 4 * 16;
@@ -247,6 +253,6 @@ struct GaParams {
 };
 
 // device error bits
-enum { ERR_BAD_LIGAND = 1, ERR_FOOTPRINT = 2, ERR_MIXED_CTA = 4 };
+enum { ERR_BAD_LIGAND = 1, ERR_FOOTPRINT = 2, ERR_MIXED_CTA = 4, ERR_STRIDE = 8 };
 
 }  // namespace adk
