@@ -234,7 +234,10 @@ typedef struct {
 } ad_ls_params;
 
 /* ADADELTA local search, one pose per warp (or per block for
- * PAPER_BASELINE), max_iters evaluations each: evaluate (E, grad) of the
+ * PAPER_BASELINE), max_iters evaluations each.  With pose_ligand != NULL and
+ * pop_per_run > 0 every run (pop_per_run consecutive poses) must belong to one
+ * ligand; CTA groups are then sized to divide pop_per_run (any population size
+ * works).  Per pose: evaluate (E, grad) of the
  * current genotype, keep it if E < best (strict; earliest wins), update every
  * gene (Z15, Z16: no angle wrapping).  On return (stream order):
  *   genes        in: start genotypes; out: best genotype per pose.

@@ -156,7 +156,10 @@ int32_t read_back_err(ad_context* ctx, cudaStream_t st) {
 int32_t opt_in_smem(ad_context* ctx, const void* k) {
     std::lock_guard<std::mutex> lock(ctx->launch_mu);
     if (std::find(ctx->smem_opted.begin(), ctx->smem_opted.end(), k) != ctx->smem_opted.end()) return AD_OK;
-    CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin));
+    cudaFuncAttributes fa;
+    CUDA_TRY(cudaFuncGetAttributes(&fa, k));  // the dynamic limit excludes the kernel's static shared memory
+    CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  ctx->max_smem_optin - (int)fa.sharedSizeBytes));
     ctx->smem_opted.push_back(k);
     return AD_OK;
 }
@@ -1897,16 +1900,6 @@ int32_t common_checks(ad_context* ctx, ad_ligand_id lig, int32_t n_poses, const 
     return AD_OK;
 }
 
-// pose_ligand launches: every ligand the launch may reference must fit the stride
-// (the kernels also check each pose's ligand on the device: ERR_STRIDE)
-int32_t check_launch_stride(ad_context* ctx, int32_t stride) {
-    int tmax = 0;
-    for_each_launch_ligand(ctx, [&](const LigSlot& o) { tmax = std::max(tmax, o.n_tors); });
-    if (stride < 6 + tmax)
-        return fail(AD_ERR_INVALID_ARG, "geno_stride %d < 6 + n_tors = %d of a ligand in the launch set", stride, 6 + tmax);
-    return AD_OK;
-}
-
 // pose_ligand launches may touch any live ligand; the scoring constants are kernel
 // parameters, so they must be identical across the live ligands
 int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
@@ -1920,7 +1913,7 @@ int32_t check_common_ff(ad_context* ctx, ad_ligand_id lig) {
 // Choose warps per CTA: the most resident warps per SM, ties -> fewer warps per CTA
 // (finer load balance across SMs).
 int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int req_warps, cudaStream_t st,
-                    bool tc_engine) {
+                    bool tc_engine, int run_align = 8) {
     if (!tc_engine) L.scratch_bytes = L.scratch_simt;
     if (p.pose_ligand)  // any ligand of the launch set may be referenced: size for the largest footprint
         for_each_launch_ligand(ctx, [&](const LigSlot& o) {
@@ -1954,7 +1947,9 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
         if (!force && pkg && !v) continue;
         for (int w = 1; w <= 32; ++w) {
             if (req_warps > 0 && w != req_warps) continue;
-            if (p.pose_ligand && ((w & (w - 1)) || w > 8)) continue;  // ad.h: ligand runs are multiples of 8
+            // pose_ligand: CTA groups never straddle two ligands' poses -- powers of two
+            // dividing the run alignment (ad.h: pop_per_run, else runs of 8)
+            if (p.pose_ligand && ((w & (w - 1)) || run_align % w)) continue;
             const size_t smem = (size_t)L.blob_bytes + (size_t)w * L.scratch_bytes;
             if (smem > (size_t)ctx->max_smem_optin) continue;
             int blocks = 0;
@@ -2020,7 +2015,6 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
     if (n_poses > 0 && !energy) return fail(AD_ERR_INVALID_ARG, "energy is NULL");
     if (pose_ligand) {
         if (int32_t rc = check_common_ff(ctx, lig)) return rc;
-        if (int32_t rc = check_launch_stride(ctx, geno_stride)) return rc;
     }
     if (int32_t rc = set_device(ctx)) return rc;
     cudaStream_t st = (cudaStream_t)stream;
@@ -2050,7 +2044,6 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
     if (n_poses > 0 && !best_energy) return fail(AD_ERR_INVALID_ARG, "best_energy is NULL");
     if (pose_ligand) {
         if (int32_t rc = check_common_ff(ctx, lig)) return rc;
-        if (int32_t rc = check_launch_stride(ctx, geno_stride)) return rc;
     }
     if (run_best && (prm->pop_per_run <= 0 || n_poses % prm->pop_per_run))
         return fail(AD_ERR_INVALID_ARG, "run_best needs pop_per_run > 0 dividing n_poses");
@@ -2099,7 +2092,17 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
         const bool wide = launch_is_wide(ctx, lig, pose_ligand);
         const WarpKernel k = p.phase_cycles ? pick_instr_kernel(prm->engine, wide)
                                             : pick_warp_kernel(prm->engine, true, true, wide);
-        if (int32_t rc = launch_warp(ctx, L, k, p, w, st, prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16))
+        // with pose_ligand and pop_per_run > 0, a ligand's poses come in whole runs
+        int align = 8;
+        if (pose_ligand && prm->pop_per_run > 0) {
+            align = 1;
+            while (align < 8 && prm->pop_per_run % (2 * align) == 0) align *= 2;
+        }
+        if (pose_ligand && w > 0 && ((w & (w - 1)) || align % w))
+            return fail(AD_ERR_INVALID_ARG, "pose_ligand launch: warps_per_cta %d must be a power of two dividing %d", w,
+                        align);
+        if (int32_t rc = launch_warp(ctx, L, k, p, w, st, prm->engine == AD_ENGINE_TC || prm->engine == AD_ENGINE_TC_FP16,
+                                     align))
             return rc;
     }
     if (run_best) {

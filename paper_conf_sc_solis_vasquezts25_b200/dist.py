@@ -38,7 +38,9 @@ def gather_records(records, group=None):
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         return records
     ws = dist.get_world_size(group)
-    out = torch.empty((ws * records.shape[0],) + tuple(records.shape[1:]), dtype=records.dtype,
-                      device=records.device)
-    dist.all_gather_into_tensor(out, records.contiguous(), group=group)
-    return out
+    src = records.contiguous()
+    if records.is_cuda and dist.get_backend(group) == "gloo":
+        src = src.cpu()  # gloo gathers host tensors (CPU tests of the multi-rank path on one GPU)
+    out = torch.empty((ws * src.shape[0],) + tuple(src.shape[1:]), dtype=src.dtype, device=src.device)
+    dist.all_gather_into_tensor(out, src, group=group)
+    return out.to(records.device)

@@ -183,7 +183,7 @@ def run_screen(ctx, grid, ff, ligands, start_genes, runs, pop, iters, rank=0, wo
     try:
         rec = s.step()
         if stream_sync:
-            torch.cuda.synchronize()
+            ctx.sync()  # device-side argument errors (pose_ligand, footprint, stride) raise here
         return rec, s.units
     finally:
         s.close()
