@@ -1,6 +1,6 @@
 #!/bin/bash
 # One GPU iteration: tests, bench lines, optional ncu captures.
-#   bash tools/gpu_round.sh TAG [tests] [smoke] [bench] [bench3] [ncu] [ncu_paper] [accuracy] [reduce] [ab] [launches]
+#   bash tools/gpu_round.sh TAG [tests] [smoke] [bench] [bench1] [bench3] [ncu] [ncu_simt] [sanitize] [ncu_paper] [accuracy] [reduce] [ab] [launches]
 #   (ab: AB_LIBS='lib1.so lib2.so ...' in the environment)
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 TAG=${1:-dev}; shift
@@ -12,6 +12,9 @@ for what in "$@"; do
       echo "pytest rc=$?" >> gpurun_out/pytest_gpu_$TAG.log; tail -4 gpurun_out/pytest_gpu_$TAG.log ;;
     smoke)
       timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_$TAG.log 2>&1; tail -2 gpurun_out/smoke_$TAG.log ;;
+    bench1)
+      timeout 900 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-paper-engine > gpurun_out/bench_${TAG}_simt.json 2>> gpurun_out/bench_$TAG.err
+      python -c "import json;d=json.load(open('gpurun_out/bench_${TAG}_simt.json'));print('simt', '%.4g'%d['value'], d['ms_per_step'], 'frac %.3f'%d['roofline']['frac'], d['clocks'])" ;;
     bench)
       for eng in tc simt; do
         timeout 900 python bench.py --steps 10 --warmup 3 --engine $eng $( [ $eng = simt ] && echo --no-cpu-baseline ) \
@@ -19,13 +22,20 @@ for what in "$@"; do
         python -c "import json;d=json.load(open('gpurun_out/bench_${TAG}_$eng.json'));print('$eng', '%.4g'%d['value'], 'frac %.3f'%d['roofline']['frac'], d['clocks'], (d.get('paper_baseline_engine') or {}).get('speedup_of_this_engine'))"
       done ;;
     bench3)
-      timeout 900 python bench.py --steps 3 --warmup 3 --config 3 --engine tc --no-cpu-baseline > gpurun_out/bench_${TAG}_cfg3.json 2>> gpurun_out/bench_$TAG.err
+      timeout 900 python bench.py --steps 3 --warmup 3 --config 3 --engine simt --no-cpu-baseline --no-paper-engine > gpurun_out/bench_${TAG}_cfg3.json 2>> gpurun_out/bench_$TAG.err
       python -c "import json;d=json.load(open('gpurun_out/bench_${TAG}_cfg3.json'));print('cfg3', '%.4g'%d['value'], 'frac %.3f'%d['roofline']['frac'], (d.get('paper_baseline_engine') or {}).get('speedup_of_this_engine'))" ;;
     ncu)
       for eng in tc simt; do
         timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_warp_engine -s 1 -c 1 \
           -o gpurun_out/prof_${eng}_$TAG python tools/prof_ls.py 2 $eng 2 > gpurun_out/ncu_${eng}_$TAG.log 2>&1
       done ;;
+    ncu_simt)
+      for cfg in 2 3; do
+        timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_warp_engine -s 1 -c 1 \
+          -o gpurun_out/prof_simt_c${cfg}_$TAG python tools/prof_ls.py $cfg simt 2 > gpurun_out/ncu_simt_c${cfg}_$TAG.log 2>&1
+      done ;;
+    sanitize)
+      bash tools/sanitize.sh $TAG ;;
     ncu_paper)
       timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_block_baseline -s 1 -c 1 \
         -o gpurun_out/prof_paper_$TAG python tools/prof_ls.py 2 paper 2 > gpurun_out/ncu_paper_$TAG.log 2>&1 ;;
