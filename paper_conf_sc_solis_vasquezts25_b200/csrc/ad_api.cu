@@ -851,9 +851,10 @@ int cherry_quarter_cost(const CherryLane* const* q, const uint8_t* flip) {
     return cost;
 }
 
-// max_steps: a schedule with more steps is not placed (steps is still reported)
+// max_steps: a schedule with more steps is not placed (steps is still reported);
+// max_K: the most gradient slots the records can address (8-bit rows, cherry_rows_fit)
 CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const std::vector<int>& pj, int effort,
-                                 int max_steps = 1 << 30) {
+                                 int max_steps = 1 << 30, int max_K = 8) {
     CherrySchedule S;
     std::vector<CherryLane> ch = make_cherries(n_idx, pi, pj);
     const int n = (int)ch.size();
@@ -869,7 +870,7 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
     std::vector<std::vector<int>> best;
     int bestK = 0;
     for (int capped = 1; capped >= 0; --capped) {
-        for (int K = 1; K <= 8; ++K) {
+        for (int K = 1; K <= max_K; ++K) {
             if (!best.empty() && (int)best.size() <= target) break;
             std::vector<std::vector<int>> steps;
             std::vector<int> rem(n), cnt(n_idx);
@@ -949,9 +950,10 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
     };
     // greedy local search (moves that do not add wavefronts), half of the moves
     // targeted at a lane on a conflicting bank group; 400k moves per step at effort 2
-    // (config 2: ~0.4 s of host time at upload), a tenth at effort 1
+    // (config 2: ~0.4 s of host time at upload), a tenth at effort 1; long schedules
+    // (global-memory cherries, config 3: 87 steps) get the budget of 24 steps
     static const long imul = getenv("AD_CHERRY_ITERS") ? atol(getenv("AD_CHERRY_ITERS")) : 400000;
-    const long iters = (long)(effort >= 2 ? imul : effort == 1 ? imul / 10 : 0) * S.steps;
+    const long iters = (long)(effort >= 2 ? imul : effort == 1 ? imul / 10 : 0) * std::min(S.steps, 24);
     uint64_t rng = 0x9E3779B97F4A7C15ull;
     int total = 0, floor_cost = 0;  // floor: 3 per quarter-warp holding a cherry
     for (int g = 0; g < NP / 8; ++g) total += qc[g];
@@ -1032,26 +1034,35 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
 }
 
 // Records of a cherry schedule (layout: ad_internal.h pka / pkb / pkc, kernel:
-// intra_cherry).  Empty ends and lanes get a zero-charge X row and a spare
+// intra_cherry).  Empty ends and lanes get a zero-charge X row and a dummy
 // gradient row in the bank group least used by that access in their
-// quarter-warp (distinct groups within a lane).  Row indices are 8-bit: X row
-// (< npad + 8) and gradient row k * npad + row (< K * npad + 8), both <= 255
+// quarter-warp (distinct groups within a lane).  distinct = true: the dummy rows
+// of one step are all different (row K * npad + r, r = group + 8 m, the smallest
+// free m), so the kernel stores unconditionally and no two lanes of a step touch
+// one row; n_spare = the spare rows that takes (a multiple of 8).  distinct =
+// false: dummies share the 8 rows K * npad + group and carry "empty" flags (a.y
+// bits 24-26) for the predicated loop (PK_PRED).  Row indices are 8-bit: X row
+// (< npad + 8) and gradient row k * npad + row (< K * npad + n_spare), both <= 255
 // (cherry_rows_fit).
 struct CherryRecords {
     std::vector<uint4> a;
     std::vector<float4> b, c;
+    int n_spare = 8;
 };
 bool cherry_rows_fit(int npad, int K) { return npad + 8 <= 256 && K * npad + 8 <= 256; }
+int cherry_max_slots(int npad) { return npad + 8 <= 256 ? std::min(8, (256 - 8) / npad) : 0; }
 
 CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector<int>& ptp,
-                            const std::vector<float4>& tp, const std::vector<float>& pdsv) {
+                            const std::vector<float4>& tp, const std::vector<float>& pdsv, bool distinct) {
     CherryRecords R;
     const size_t n = (size_t)S.steps * 32;
     R.a.resize(n);
     R.b.resize(n);
     R.c.resize(n);
     const int K = S.slots;
+    uint64_t step_used[4] = {0, 0, 0, 0};  // dummy rows (0..255) taken in the current step
     for (size_t q0 = 0; q0 < n; q0 += 8) {  // one quarter-warp
+        if (q0 % 32 == 0) step_used[0] = step_used[1] = step_used[2] = step_used[3] = 0;
         int cnt[3][8] = {};
         for (size_t q = q0; q < q0 + 8; ++q) {
             const CherryLane& L = S.lane[q];
@@ -1071,7 +1082,13 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector
                 taken |= 1u << r;
                 cnt[acc][r]++;
                 xr[acc] = (uint32_t)(npad + r);
-                gr[acc] = (uint32_t)(K * npad + r);
+                int row = r;
+                if (distinct) {
+                    while (step_used[row >> 6] >> (row & 63) & 1u) row += 8;  // (< 256: at most 96 per step)
+                    step_used[row >> 6] |= 1ull << (row & 63);
+                    R.n_spare = std::max(R.n_spare, (row + 8) & ~7);
+                }
+                gr[acc] = (uint32_t)(K * npad + row);
             };
             if (L.c >= 0) {
                 xr[0] = (uint32_t)L.c;
@@ -1101,7 +1118,10 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector
             uint32_t d0, d1;
             memcpy(&d0, &dsv[0], 4);
             memcpy(&d1, &dsv[1], 4);
-            R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16), gr[0] | (gr[1] << 8) | (gr[2] << 16), d0, d1);
+            // a.y bits 24-26: the centre / end 0 / end 1 is empty (PK_PRED: the kernel skips its store)
+            const uint32_t fl = (L.c < 0 ? 1u : 0u) | (L.c < 0 || L.e[0] < 0 ? 2u : 0u) | (L.c < 0 || L.e[1] < 0 ? 4u : 0u);
+            R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16),
+                                gr[0] | (gr[1] << 8) | (gr[2] << 16) | (fl << 24), d0, d1);
             R.b[q] = make_float4(cA[0], cA[1], cB[0], cB[1]);
             R.c[q] = make_float4(r0[0], r0[1], cC[0], cC[1]);
         }
@@ -1558,7 +1578,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     Schedule sch;
     OwnerList own;
     CherrySchedule cs;
-    bool cherry = false;
+    bool cherry = false, cherry_gm = false;
     if (mode == INTRA_OWNER) {
         own = build_owner(N, pi, pj, ptp, pd);
         if (own.C * 32 > 65535) return fail(AD_ERR_LIMIT, "too many owner chunks");
@@ -1585,16 +1605,27 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         }
         // the cherry schedule when it fits shared memory (its records and the prec
         // list) and its row offsets fit 16 bits; else the pair-step schedule
-        if (ctx->pk_smem_max > 0 && P > 0) {
+        // A cherry schedule too long for shared memory streams its records from global
+        // memory instead (cherry_gm: intra_cherry_gm, 128-register kernels); the 8-bit
+        // row indices cap the gradient slots (cherry_max_slots).  AD_PK_SMEM_MAX=0 turns
+        // cherries off altogether, AD_CHERRY_GM=0 the global-memory variant (A/B knobs).
+        static const bool gm_on = !getenv("AD_CHERRY_GM") || atoi(getenv("AD_CHERRY_GM")) != 0;
+        const int max_K = cherry_max_slots(npad_of(N));
+        if (ctx->pk_smem_max > 0 && P > 0 && max_K > 0) {
             const int max_steps = std::min(ctx->pairs_smem_max / (kPairsPerStep * 12), ctx->pk_smem_max / (kLanes * 48));
-            cs = schedule_cherries(npad_of(N), si, sj, ctx->sched_effort, max_steps);
-            cherry = cs.steps <= max_steps && cherry_rows_fit(npad_of(N), cs.slots);
+            cs = schedule_cherries(npad_of(N), si, sj, ctx->sched_effort, gm_on ? (1 << 30) : max_steps, max_K);
+            const bool fit = cherry_rows_fit(npad_of(N), cs.slots);
+            cherry = cs.steps <= max_steps && fit;
+            cherry_gm = !cherry && fit && gm_on;
         }
         // the prec list (the paper-style baseline's pairs; the warp engine's schedule
         // when it runs no cherries) is the pair-step schedule either way, so the
         // baseline is the same program with or without cherries
         sch = schedule_pairs(N, si, sj, ptp, pd, pcq, ctx->sched_effort);
-        if (cherry && (int64_t)(sch.rec.size() + sch.dsv.size()) * 4 > ctx->pairs_smem_max) cherry = false;
+        if (cherry && (int64_t)(sch.rec.size() + sch.dsv.size()) * 4 > ctx->pairs_smem_max) {
+            cherry = false;
+            cherry_gm = gm_on;
+        }
     }
     if (own.comb.empty()) own.comb.assign(N, make_int2(0, 0));
 
@@ -1696,14 +1727,24 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
         h.off_combidx = B.put(own.combidx.data(), sizeof(uint16_t) * own.combidx.size());
         o.ws = warp_scratch_layout(N, T, h.n_slots, own.C);
         if (warp_cherry) {
-            // cherry records (ad_internal.h pka / pkb / pkc), staged with the tables
-            const CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd);
+            // cherry records (ad_internal.h pka / pkb / pkc), staged with the tables (or,
+            // cherry_gm, left in global memory).  Distinct dummy rows when they fit the
+            // 8-bit row indices and at most 32 spare rows (512 B per warp), else shared
+            // dummies with predicated stores (PK_PRED).
+            CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, true);
+            h.pk_flags = cherry_gm ? PK_GMEM : 0;
+            if (cs.slots * h.n_pad + cr.n_spare > 256 || cr.n_spare > 32) {
+                cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, false);
+                h.pk_flags |= PK_PRED;
+            }
+            o.ws = warp_scratch_layout(N, T, h.n_slots, own.C, cr.n_spare);
             h.off_tp = h.off_prec = h.off_pdsv = h.off_pkg = 0;
             h.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
             B.put(cr.b.data(), sizeof(float4) * cr.b.size());
             B.put(cr.c.data(), sizeof(float4) * cr.c.size());
-            h.pairs_gmem = 0;
-            h.blob_bytes = h.stage_bytes = (int32_t)B.buf.size();
+            h.pairs_gmem = cherry_gm ? 1 : 0;  // (cherry_gm: records after the staged prefix)
+            h.blob_bytes = (int32_t)B.buf.size();
+            h.stage_bytes = cherry_gm ? h.off_pk : h.blob_bytes;
         } else {
             // 8 copies of every entry, copy c at index t*8 + c: lane l reads copy l % 8,
             // so the 8 lanes of a quarter-warp always hit 8 different bank groups.
@@ -1733,7 +1774,8 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
                     const uint32_t gi = (uint32_t)o.ws.g + 16u * (si * npad + i);
                     const uint32_t gj = (uint32_t)o.ws.g + 16u * (sj * npad + j);
                     if ((int)si == sch.slots) {  // empty place: zero-charge rows, zero coefficients, spare row
-                        pka[q] = make_uint4((16u * npad) | ((16u * (npad + 1)) << 16), gi | (gj << 16), 0u, 0u);
+                        // bit 15 of the i offset marks the empty place (X offsets < 2^13)
+                        pka[q] = make_uint4((16u * npad) | 0x8000u | ((16u * (npad + 1)) << 16), gi | (gj << 16), 0u, 0u);
                         pkb[q] = make_float2(0.f, 1.f);
                         continue;
                     }
@@ -1759,8 +1801,9 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     };
     const Built base = build_blob(false);
     Built warp;
-    if (cherry) warp = build_blob(true);
-    const Built& W = cherry ? warp : base;
+    const bool two = cherry || cherry_gm;
+    if (two) warp = build_blob(true);
+    const Built& W = two ? warp : base;
 
     std::lock_guard<std::mutex> lock(ctx->mu);
     if (int32_t rc = set_device(ctx)) return rc;
@@ -1772,12 +1815,12 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     s.block_scratch = block_scratch_layout(N, T, 0).bytes;
     s.n_atoms = N;
     s.n_tors = T;
-    s.pkg = W.h.off_pkg != 0 && 6 + T > 32;
+    s.pkg = (W.h.off_pkg != 0 && 6 + T > 32) || (W.h.pk_flags & PK_GMEM);  // runs on the 128-register kernels
     memcpy(s.ff, H.ff, sizeof(s.ff));
     CUDA_TRY(cudaMalloc(&s.d_blob, W.buf.size()));
     CUDA_TRY(cudaMemcpy(s.d_blob, W.buf.data(), W.buf.size(), cudaMemcpyHostToDevice));
     s.d_base = s.d_blob;
-    if (cherry) {
+    if (two) {
         if (cudaMalloc(&s.d_base, base.buf.size()) != cudaSuccess) {
             cudaFree(s.d_blob);
             return fail(AD_ERR_OOM, "ligand blob allocation failed");
@@ -1936,15 +1979,15 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     struct Cand { int w = 0, active = -1; double cost = 1e300; size_t sm_smem = 0; size_t smem = 0; WarpKernelFn k = nullptr; };
     Cand pick;
     static const int force = getenv("AD_MAXREG") ? atoi(getenv("AD_MAXREG")) : 0;  // A/B knob: 80 or 128
-    // ligands with pre-decoded global-memory schedules run the 128-register kernels,
-    // which alone carry that loop (config 3: 121.0 ms vs 130.6 ms on the 80-register
-    // kernels' record-decoding loop)
+    // ligands with global-memory schedules (pre-decoded places of wide ligands, streamed
+    // cherry records) run the 128-register kernels, which alone carry those loops
+    // (config 3: 121.0 ms vs 130.6 ms on the 80-register kernels' record-decoding loop)
     bool pkg = L.pkg;
     if (p.pose_ligand) for_each_launch_ligand(ctx, [&](const LigSlot& o) { pkg |= o.pkg; });
     for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
         if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
-        if (!force && pkg && !v) continue;
+        if (pkg && !v) continue;
         for (int w = 1; w <= 32; ++w) {
             if (req_warps > 0 && w != req_warps) continue;
             // pose_ligand: CTA groups never straddle two ligands' poses -- powers of two
@@ -2338,7 +2381,7 @@ int32_t adx_debug_cherries(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
     }
     if (out_atom_slot)
         for (int a = 0; a < n_atoms; ++a) out_atom_slot[a] = slot[a];
-    const CherrySchedule S = schedule_cherries(npad_of(n_atoms), pi, pj, effort);
+    const CherrySchedule S = schedule_cherries(npad_of(n_atoms), pi, pj, effort, 1 << 30, cherry_max_slots(npad_of(n_atoms)));
     *out_steps = S.steps;
     *out_slots = S.slots;
     if (out)

@@ -71,6 +71,11 @@ enum {
 //                  conflict-free read-modify-write as in INTRA_SCATTER (half the
 //                  shared-memory RMW traffic, no duplicated flops).
 enum { INTRA_SCATTER = 0, INTRA_OWNER = 1, INTRA_HYBRID = 2 };
+// LigHeader.pk_flags: PK_GMEM = the cherry records stay in global memory (not staged;
+// intra_cherry_gm, 128-register kernels); PK_PRED = empty ends share dummy gradient
+// rows with other lanes of their step, so their stores are predicated off (else every
+// dummy target of a step is a distinct row and the loop stores unconditionally).
+enum { PK_GMEM = 1, PK_PRED = 2 };
 // owner-mode entry: a | b<<8 | tp<<16 | flags<<24
 enum { OF_PRIMARY = 1, OF_FIRST = 2, OF_LAST = 4, OF_DUMMY = 8 };
 
@@ -87,9 +92,10 @@ struct alignas(16) LigHeader {
                                                         //      off_pk: cherry records (0 = none); base_*: steps
                                                         //      and slots of the prec list (= n_rounds / n_slots
                                                         //      unless the warp engine runs a cherry schedule)
-    int32_t off_pkg, off_tors64, ws_trig64, reserved3;  // 160  off_pkg: pre-decoded global-memory places (0 = none);
+    int32_t off_pkg, off_tors64, ws_trig64, pk_flags;   // 160  off_pkg: pre-decoded global-memory places (0 = none);
                                                         //      off_tors64: double [T][6] axis point P_b, unit axis u_b
-                                                        //      (the FP64 torsion chain); ws_trig64: per-warp double2 [T]
+                                                        //      (the FP64 torsion chain); ws_trig64: per-warp double2 [T];
+                                                        //      pk_flags (PK_*): how the cherry loop runs
     float ff[FF_N];                                     // 224
 };
 static_assert(sizeof(LigHeader) == 224, "header size");
@@ -140,7 +146,7 @@ struct WarpScratch {
 __host__ __device__ inline int32_t align16(int32_t v) { return (v + 15) & ~15; }
 
 __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int32_t n_tors, int32_t n_slots,
-                                                           int32_t n_chunks) {
+                                                           int32_t n_chunks, int32_t n_spare = 8) {
     WarpScratch s;
     const int32_t npad = (n_atoms + 7) & ~7;
     const int32_t mpad = (n_tors + 1 + 15) / 16 * 16;
@@ -148,9 +154,10 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     // X rows + 8 zero-charge rows (positions (r,0,0), bank group r) that the empty
     // ends of cherry schedules read
     s.x = o;     o += 16 * (npad + 8);
-    // rows of npad float4 (slot k of atom a at k * npad + a) + the start of a spare
-    // row K: empty schedule places only ever target K * npad + (0..7)
-    s.g = o;     o += 16 * npad * n_slots + 16 * 8;
+    // rows of npad float4 (slot k of atom a at k * npad + a) + n_spare spare rows
+    // K * npad + (0..n_spare-1): the targets of empty schedule places (8, or the
+    // distinct dummy rows of a cherry schedule without PK_PRED)
+    s.g = o;     o += 16 * npad * n_slots + 16 * n_spare;
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.trig64 = o; o += 16 * n_tors;
     s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);

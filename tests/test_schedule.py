@@ -99,17 +99,20 @@ def _cherries(lib, n_atoms, pairs, effort=2):
     return steps.value, slots.value, out[:steps.value * 32], slot[:n_atoms]
 
 
-@pytest.mark.parametrize("n_atoms,n_tors,seed", [(12, 2, 1), (40, 8, 2), (65, 16, 6), (20, 0, 7)])
+@pytest.mark.parametrize("n_atoms,n_tors,seed", [(12, 2, 1), (40, 8, 2), (65, 16, 6), (20, 0, 7), (110, 32, 3)])
 def test_cherries_cover_pairs_with_distinct_targets(lib, n_atoms, n_tors, seed):
     """Every pair is one end of exactly one cherry (c; e0, e1) whose two pairs share
     the centre c; per step the gradient targets (slot, row) of all centres and ends
-    are distinct (the kernel's read-modify-writes are race-free without atomics)."""
-    L = synth.make_ligand(seed, n_atoms, n_tors, 8, chainlike=False)
+    are distinct (the kernel's read-modify-writes are race-free without atomics).
+    (110, 32): config 3's shape, whose 87-step schedule streams from global memory;
+    the 8-bit row indices of the records cap the slots at K npad + 8 <= 256."""
+    L = synth.make_ligand(seed, n_atoms, n_tors, 8, chainlike=n_atoms > 80)
     R, K, o, slot = _cherries(lib, L.n_atoms, L.pairs)
     npad = (L.n_atoms + 7) & ~7
     c, e, p, k = o[:, 0], o[:, 1:3], o[:, 3:5], o[:, 5:8]
     live = c >= 0
     assert 1 <= K <= 8 and np.all(k[live][:, 0] < K)
+    assert K * npad + 8 <= 256
     got = []
     for lane in np.nonzero(live)[0]:
         for t in range(2):
