@@ -136,7 +136,7 @@ struct WarpScratch {
     int32_t d;      // float  [Mpad][8]     D = M_ext W (TC)
     int32_t trig;   // float2 [T+3]         cos, sin of torsion angles, then phi, theta, alpha/2
     int32_t trig64; // double2 [T]          sin, 1 - cos of torsion angles in FP64 (the chain)
-    int32_t tw;     // float4 [T][2]        world torsion axis u_b and X_{a_b}
+    int32_t tw;     // float4 [6 + T][2]    per-gene gradient vectors U_k, W_k (.w: sum rows)
     int32_t genes;  // float  [64]
     int32_t part;   // float4 [C][32]       owner mode: per-(lane, chunk) partial gradients
     int32_t bytes_simt;
@@ -160,7 +160,7 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     s.g = o;     o += 16 * npad * n_slots + 16 * n_spare;
     s.trig = o;  o += align16(8 * (n_tors + 3));  // torsions, then phi, theta, alpha/2
     s.trig64 = o; o += 16 * n_tors;
-    s.tw = o;    o += 32 * (n_tors > 0 ? n_tors : 1);
+    s.tw = o;    o += 32 * (6 + n_tors);  // per-gene gradient vectors (U, W) + rows
     s.genes = o; o += 4 * kMaxGenes;
     s.part = o;  o += 16 * 32 * n_chunks;
     // the SIMT engine needs neither W nor D: its prefix sums overwrite the X and
