@@ -88,6 +88,33 @@ TYPE_PARAMS = {
     "Cl": (4.09, 0.276, 35.8235, -0.00110, 0, 0.0, 0.0),
 }
 
+def pair_coefficients(names, params=None) -> np.ndarray:
+    """Type-pair table [nt, nt, 5] = (cA, cB, r0, m, n) of the AD4 pair forms [ext]:
+    donor-H x acceptor pairs 12-10 at (Rhb, eps_hb) of the acceptor, every other
+    pair 12-6 at R = (R_i + R_j) / 2, eps = sqrt(eps_i eps_j); cA = fe eps r0^m n /
+    (m - n), cB = fe eps r0^n m / (m - n) (minimum -fe eps at r0); FE weights folded
+    in.  An input table (the ABI's tp_coef), not method arithmetic."""
+    params = TYPE_PARAMS if params is None else params
+    nt = len(names)
+    tp = np.zeros((nt, nt, 5), dtype=np.float64)
+    for a, na in enumerate(names):
+        for b, nb in enumerate(names):
+            Ra, ea, _, _, rola, Rhba, ehba = params[na]
+            Rb, eb, _, _, rolb, Rhbb, ehbb = params[nb]
+            if (rola, rolb) in ((1, 2), (2, 1)):
+                r0, eps = (Rhbb, ehbb) if rola == 1 else (Rhba, ehba)
+                m, n = 12.0, 10.0
+                fe = FE_COEFF_HBOND
+            else:
+                r0, eps = 0.5 * (Ra + Rb), np.sqrt(ea * eb)
+                m, n = 12.0, 6.0
+                fe = FE_COEFF_VDW
+            cA = fe * eps * r0 ** m * n / (m - n)
+            cB = fe * eps * r0 ** n * m / (m - n)
+            tp[a, b] = (cA, cB, r0, m, n)
+    return tp
+
+
 TYPESETS = {
     3: ["C", "OA", "HD"],
     6: ["C", "A", "N", "NA", "OA", "HD"],
@@ -347,23 +374,7 @@ def make_ligand(seed: int, n_atoms: int, n_tors: int, n_types: int,
 
     xyz = xyz - xyz.mean(axis=0)
 
-    nt = len(names)
-    tp = np.zeros((nt, nt, 5), dtype=np.float64)
-    for a, na in enumerate(names):
-        for b, nb in enumerate(names):
-            Ra, ea, _, _, rola, Rhba, ehba = TYPE_PARAMS[na]
-            Rb, eb, _, _, rolb, Rhbb, ehbb = TYPE_PARAMS[nb]
-            if (rola, rolb) in ((1, 2), (2, 1)):
-                r0, eps = (Rhbb, ehbb) if rola == 1 else (Rhba, ehba)
-                m, n = 12.0, 10.0
-                fe = FE_COEFF_HBOND
-            else:
-                r0, eps = 0.5 * (Ra + Rb), np.sqrt(ea * eb)
-                m, n = 12.0, 6.0
-                fe = FE_COEFF_VDW
-            cA = fe * eps * r0 ** m * n / (m - n)
-            cB = fe * eps * r0 ** n * m / (m - n)
-            tp[a, b] = (cA, cB, r0, m, n)
+    tp = pair_coefficients(names)
     return Ligand(
         ref_xyz=xyz.astype(np.float32),
         atom_map=atom_type.copy(),
