@@ -914,6 +914,46 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
     S.steps = (int)best.size();
     S.slots = bestK;
     if (S.steps > max_steps) return S;
+    {   // spread the empty lanes: first-fit leaves them all in the last steps, where their
+        // dummy gradient targets cannot all get distinct rows (pack_cherries); move cherries
+        // from full steps into deficient ones (within K) until every step holds at least
+        // 32 - ceil(empty / steps) cherries
+        const int n_empty = S.steps * 32 - n, lo = 32 - (n_empty + S.steps - 1) / S.steps;
+        std::vector<int> c2((size_t)S.steps * n_idx, 0);
+        for (int st = 0; st < S.steps; ++st)
+            for (int x : best[st]) {
+                const CherryLane& L = ch[x];
+                c2[(size_t)st * n_idx + L.c]++;
+                for (int k = 0; k < 2; ++k)
+                    if (L.e[k] >= 0) c2[(size_t)st * n_idx + L.e[k]]++;
+            }
+        auto fits_in = [&](int st, const CherryLane& L) {
+            if (c2[(size_t)st * n_idx + L.c] >= bestK) return false;
+            for (int k = 0; k < 2; ++k)
+                if (L.e[k] >= 0 && c2[(size_t)st * n_idx + L.e[k]] >= bestK) return false;
+            return true;
+        };
+        auto move = [&](int from, size_t idx, int to) {
+            const int x = best[from][idx];
+            const CherryLane& L = ch[x];
+            for (int k = -1; k < 2; ++k) {
+                const int a = k < 0 ? L.c : L.e[k];
+                if (a < 0) continue;
+                c2[(size_t)from * n_idx + a]--;
+                c2[(size_t)to * n_idx + a]++;
+            }
+            best[to].push_back(x);
+            best[from].erase(best[from].begin() + (long)idx);
+        };
+        for (int to = 0; to < S.steps; ++to) {
+            for (int from = 0; from < S.steps && (int)best[to].size() < lo; ++from) {
+                if (from == to) continue;
+                for (size_t i = 0; i < best[from].size() && (int)best[from].size() > lo && (int)best[to].size() < lo;) {
+                    if (fits_in(to, ch[best[from][i]])) move(from, i, to); else ++i;
+                }
+            }
+        }
+    }
     S.lane.assign((size_t)S.steps * 32, CherryLane{});
     // (3) placement: one local search over all positions (swaps within and across
     // steps that keep every step within K targets per atom, and end flips)
@@ -1733,7 +1773,9 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             // dummies with predicated stores (PK_PRED).
             CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, true);
             h.pk_flags = cherry_gm ? PK_GMEM : 0;
-            if (cs.slots * h.n_pad + cr.n_spare > 256 || cr.n_spare > 32) {
+            // (global-memory cherries always take the predicated loop: measured faster than
+            // distinct dummies on config 3, 114.1 vs 120.4 ms per LS launch)
+            if (cherry_gm || cs.slots * h.n_pad + cr.n_spare > 256 || cr.n_spare > 32) {
                 cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, false);
                 h.pk_flags |= PK_PRED;
             }
