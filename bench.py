@@ -601,6 +601,45 @@ def main():
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_val = (w.n_poses if strong else world * n) * w.iters / (float(e2e_t.item()) / 1e3)
 
+    # ---- config 1 (BASELINE configs[0]): ONE ad_score_poses call (256 poses, energy + gradient)
+    # end to end with host buffers -- pinned H2D of the genotypes, the call, D2H of energies and
+    # gradients, synchronize -- timed on the host clock per call (the latency a GA driver sees) ----
+    call1 = None
+    if rank == 0:
+        w1 = synth.make_config(1)
+        ctx1 = ad.Context(local)
+        try:
+            ctx1.upload_grid(w1.grid)
+            lid1 = ctx1.upload_ligand(w1.ligands[0], w1.ff)
+            hg1 = torch.from_numpy(np.ascontiguousarray(w1.genes)).pin_memory()
+            g1 = torch.empty_like(hg1, device=dev)
+            n1, s1 = hg1.shape
+            out1 = torch.empty(n1 * (1 + s1), device=dev)  # energies then gradients: ONE D2H copy
+            E1, G1 = out1[:n1], out1[n1:].view(n1, s1)
+            hout1 = torch.empty(n1 * (1 + s1)).pin_memory()
+            host_us, dev_us = [], []
+            for k in range(230):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                t0 = time.perf_counter()
+                a.record(stream)
+                g1.copy_(hg1, non_blocking=True)
+                ad.ad_score_poses(ctx1.h, lid1, None, g1, E1, G1)
+                hout1.copy_(out1, non_blocking=True)
+                b.record(stream)
+                b.synchronize()
+                t1 = time.perf_counter()
+                if k >= 30:
+                    host_us.append((t1 - t0) * 1e6)
+                    dev_us.append(a.elapsed_time(b) * 1e3)
+            call1 = {"workload": f"{w1.name}: {w1.n_poses} poses, energy + gene gradient, one ad_score_poses call",
+                     "us_per_call_host_median": statistics.median(host_us),
+                     "us_per_call_device_median": statistics.median(dev_us),
+                     "evals_per_s_e2e": w1.n_poses / (statistics.median(host_us) / 1e6),
+                     "h2d_bytes": int(hg1.numel() * 4), "d2h_bytes": int(hout1.numel() * 4),
+                     "calls": len(host_us)}
+        finally:
+            ctx1.close()
+
     # ---- paper-style block-per-pose engines, same workload (the self-built speedup denominator) ----
     paper = None
     if rank == 0 and not args.no_paper_engine and not args.engine.startswith("paper"):
@@ -657,6 +696,7 @@ def main():
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h_genes.numel() * 4),
                     "d2h_bytes_per_step": int((h_bestE.numel() + h_run.numel()) * 4)},
             "clocks": ck, "gpu_launches": 2 * args.steps,
+            "config1_score_call": call1,
             "paper_baseline_engine": paper,
         }
         print(json.dumps(line), flush=True)

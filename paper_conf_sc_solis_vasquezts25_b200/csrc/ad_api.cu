@@ -83,15 +83,35 @@ struct ad_context {
     LigDev* d_ligtab = nullptr;
     int32_t ligtab_cap = 0;
     int32_t* d_err = nullptr;
-    // device error word read back asynchronously: after every launch a 4-byte copy
-    // d_err -> h_err (pinned) and an event on the caller's stream; later calls
-    // report it once the event has completed (no host-device synchronisation)
+    // device error word: kernels atomicOr their ERR_* bits into d_err (device memory)
+    // and, on that rare path only, store the bits they saw into h_err, a mapped pinned
+    // host word (d_err_seen is its device address).  After every call an event is
+    // recorded on the caller's stream; a later call reads h_err once the event has
+    // completed -- no copy and no host-device synchronisation on the normal path --
+    // and, if it is set, copies the complete d_err synchronously and reports it.
     int32_t* h_err = nullptr;
+    int32_t* d_err_seen = nullptr;
     cudaEvent_t err_ev = nullptr;
     bool err_pending = false;
     // launch-shape caches: cudaFuncSetAttribute once per kernel, occupancy per
     // (kernel, threads, dynamic shared memory)
     std::mutex launch_mu;
+    // launch_warp decisions: key (kernels, footprint, n_poses, request) -> (W, kernel, smem)
+    struct LaunchKey {
+        const void *lo, *hi;
+        int32_t blob, scratch, n_poses, req, mixed, align, pkg;
+        bool operator==(const LaunchKey& o) const {
+            return lo == o.lo && hi == o.hi && blob == o.blob && scratch == o.scratch && n_poses == o.n_poses &&
+                   req == o.req && mixed == o.mixed && align == o.align && pkg == o.pkg;
+        }
+    };
+    struct LaunchPick {
+        LaunchKey key;
+        int w;
+        const void* k;
+        size_t smem;
+    };
+    std::vector<LaunchPick> launch_cache;
     std::vector<const void*> smem_opted;
     std::vector<std::array<long long, 4>> occ;  // {kernel, threads, smem, blocks}
     // AD_INTRA_MODE=owner|scatter at context creation (tuning knob; scatter measured
@@ -114,6 +134,8 @@ struct ad_context {
 namespace {
 
 int32_t set_device(ad_context* ctx) {
+    int cur = -1;
+    if (cudaGetDevice(&cur) == cudaSuccess && cur == ctx->device) return AD_OK;
     CUDA_TRY(cudaSetDevice(ctx->device));
     return AD_OK;
 }
@@ -135,18 +157,17 @@ int32_t check_device_err(ad_context* ctx, cudaStream_t st) {
     if (q == cudaErrorNotReady) return AD_OK;
     if (q != cudaSuccess) return fail(AD_ERR_CUDA, "error read-back: %s", cudaGetErrorString(q));
     ctx->err_pending = false;
-    const int32_t h = *ctx->h_err;
-    if (h) {
-        *ctx->h_err = 0;
-        CUDA_TRY(cudaMemsetAsync(ctx->d_err, 0, sizeof(int32_t), st));
-        return report_device_err(h);
-    }
-    return AD_OK;
+    if (*reinterpret_cast<volatile int32_t*>(ctx->h_err) == 0) return AD_OK;
+    // an error was flagged: the complete bits from the device word (rare path)
+    int32_t h = 0;
+    CUDA_TRY(cudaMemcpy(&h, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemset(ctx->d_err, 0, sizeof(int32_t)));
+    *reinterpret_cast<volatile int32_t*>(ctx->h_err) = 0;
+    return report_device_err(h ? h : ERR_FOOTPRINT);
 }
 
-// Enqueue the read-back of the device error word after this call's launches.
+// Mark this call's launches for the error check of a later call (an event only).
 int32_t read_back_err(ad_context* ctx, cudaStream_t st) {
-    CUDA_TRY(cudaMemcpyAsync(ctx->h_err, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
     CUDA_TRY(cudaEventRecord(ctx->err_ev, st));
     ctx->err_pending = true;
     return AD_OK;
@@ -1381,8 +1402,9 @@ int32_t ad_context_create(int32_t cuda_device, ad_context** out) {
         e = cudaDeviceGetAttribute(&ctx->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, cuda_device);
     if (e == cudaSuccess) e = cudaMalloc(&ctx->d_err, sizeof(int32_t));
     if (e == cudaSuccess) e = cudaMemset(ctx->d_err, 0, sizeof(int32_t));
-    if (e == cudaSuccess) e = cudaHostAlloc(reinterpret_cast<void**>(&ctx->h_err), sizeof(int32_t), cudaHostAllocDefault);
+    if (e == cudaSuccess) e = cudaHostAlloc(reinterpret_cast<void**>(&ctx->h_err), sizeof(int32_t), cudaHostAllocMapped);
     if (e == cudaSuccess) *ctx->h_err = 0;
+    if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&ctx->d_err_seen), ctx->h_err, 0);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->err_ev, cudaEventDisableTiming);
     if (e != cudaSuccess) {
         delete ctx;
@@ -2026,6 +2048,29 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // (config 3: 121.0 ms vs 130.6 ms on the 80-register kernels' record-decoding loop)
     bool pkg = L.pkg;
     if (p.pose_ligand) for_each_launch_ligand(ctx, [&](const LigSlot& o) { pkg |= o.pkg; });
+    // the decision depends on nothing else: cached (a config-1 score call is ~9 us of
+    // kernel; the 64-candidate search must not add to it on every call)
+    const ad_context::LaunchKey key{reinterpret_cast<const void*>(kern.lo), reinterpret_cast<const void*>(kern.hi),
+                                    L.blob_bytes, L.scratch_bytes, p.n_poses, req_warps, p.pose_ligand ? 1 : 0,
+                                    run_align, pkg ? 1 : 0};
+    {
+        std::lock_guard<std::mutex> lock(ctx->launch_mu);
+        for (const auto& e : ctx->launch_cache)
+            if (e.key == key) {
+                p.smem_blob = L.blob_bytes;
+                p.smem_scratch = L.scratch_bytes;
+                const int grid = (p.n_poses + e.w - 1) / e.w;
+                const WarpKernelFn k = reinterpret_cast<WarpKernelFn>(const_cast<void*>(e.k));
+                k<<<grid, e.w * 32, e.smem, st>>>(p);
+                ctx->last_maxreg = k == kern.hi ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG;
+                ctx->last_grid = grid;
+                ctx->last_block = e.w * 32;
+                ctx->last_smem = (int32_t)e.smem;
+                CUDA_TRY(cudaGetLastError());
+                return AD_OK;
+            }
+    }
+    static const bool debug_launch = getenv("AD_DEBUG_LAUNCH") != nullptr;
     for (int v = 0; v < 2; ++v) {
         const WarpKernelFn k = v ? kern.hi : kern.lo;
         if (force && force != (v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG)) continue;
@@ -2047,7 +2092,7 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             const double g1 = 1.0 - 0.48;
             double cost = (double)full * std::pow((double)active, g1) + (rem ? std::pow((double)(rem * w), g1) : 0.0);
             if (v) cost *= 0.85;
-            if (getenv("AD_DEBUG_LAUNCH"))
+            if (debug_launch)
                 fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld per_sm=%ld cost=%.3f\n",
                         v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, per_sm, cost);
             const size_t sm_smem = (size_t)std::min<long>(blocks, per_sm) * smem;  // in use on the busiest SM
@@ -2064,6 +2109,11 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
                     L.scratch_bytes);
     p.smem_blob = L.blob_bytes;
     p.smem_scratch = L.scratch_bytes;
+    {
+        std::lock_guard<std::mutex> lock(ctx->launch_mu);
+        if (ctx->launch_cache.size() < 4096)
+            ctx->launch_cache.push_back({key, best_w, reinterpret_cast<const void*>(best_k), best_smem});
+    }
     const int grid = (p.n_poses + best_w - 1) / best_w;
     best_k<<<grid, best_w * 32, best_smem, st>>>(p);
     ctx->last_maxreg = best_k == kern.hi ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG;
@@ -2083,6 +2133,7 @@ KParams base_params(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligan
     p.n_poses = n_poses;
     p.stride = stride;
     p.err = ctx->d_err;
+    p.err_seen = ctx->d_err_seen;
     p.n_ligs = (int32_t)ctx->ligs.size();
     p.max_iters = 1;
     p.pc = pair_const_from_ff(ctx->ligs[lig].ff);
@@ -2455,7 +2506,7 @@ int32_t ad_sync(ad_context* ctx, void* stream) {
     int32_t h = 0;
     CUDA_TRY(cudaMemcpy(&h, ctx->d_err, sizeof(int32_t), cudaMemcpyDeviceToHost));
     ctx->err_pending = false;
-    *ctx->h_err = 0;
+    *reinterpret_cast<volatile int32_t*>(ctx->h_err) = 0;
     if (h) {
         CUDA_TRY(cudaMemset(ctx->d_err, 0, sizeof(int32_t)));
         return report_device_err(h);

@@ -239,7 +239,8 @@ struct KParams {
     float* aux;
     float* trace;
     int64_t* n_evals;
-    int32_t* err;
+    int32_t* err;        // device error word (ERR_* bits, atomicOr)
+    int32_t* err_seen;   // mapped pinned host word: set on the (rare) error path only
     int32_t max_iters;
     float rho, eps;
     int32_t smem_blob;      // bytes reserved for the blob in shared memory
