@@ -1012,9 +1012,9 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
     // greedy local search (moves that do not add wavefronts), half of the moves
     // targeted at a lane on a conflicting bank group; 400k moves per step at effort 2
     // (config 2: ~0.4 s of host time at upload), a tenth at effort 1; long schedules
-    // (global-memory cherries, config 3: 87 steps) get the budget of 24 steps
+    // (global-memory cherries, config 3: 89 steps) get the budget of 48 steps
     static const long imul = getenv("AD_CHERRY_ITERS") ? atol(getenv("AD_CHERRY_ITERS")) : 400000;
-    const long iters = (long)(effort >= 2 ? imul : effort == 1 ? imul / 10 : 0) * std::min(S.steps, 24);
+    const long iters = (long)(effort >= 2 ? imul : effort == 1 ? imul / 10 : 0) * std::min(S.steps, 48);
     uint64_t rng = 0x9E3779B97F4A7C15ull;
     int total = 0, floor_cost = 0;  // floor: 3 per quarter-warp holding a cherry
     for (int g = 0; g < NP / 8; ++g) total += qc[g];
@@ -1059,8 +1059,22 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
         if (sa != sb && (!fits(sa, pos[b], pos[a]) || !fits(sb, pos[a], pos[b]))) continue;
         std::swap(pos[a], pos[b]);
         std::swap(flip[a], flip[b]);
-        const int ca = cherry_quarter_cost(&pos[8 * ga], &flip[8 * ga]);
-        const int cb = cherry_quarter_cost(&pos[8 * gb], &flip[8 * gb]);
+        // the moved cherries take their best end orientation at the new positions
+        int ca = 0, cb = 0;
+        const uint8_t fa0 = flip[a], fb0 = flip[b];
+        {
+            int best_c = 1 << 30;
+            uint8_t bfa = fa0, bfb = fb0;
+            for (int m = 0; m < 4; ++m) {
+                flip[a] = fa0 ^ (uint8_t)(m & 1);
+                flip[b] = fb0 ^ (uint8_t)(m >> 1);
+                const int x = cherry_quarter_cost(&pos[8 * ga], &flip[8 * ga]);
+                const int y = cherry_quarter_cost(&pos[8 * gb], &flip[8 * gb]);
+                if (x + y < best_c) { best_c = x + y; ca = x; cb = y; bfa = flip[a]; bfb = flip[b]; }
+            }
+            flip[a] = bfa;
+            flip[b] = bfb;
+        }
         if (ca + cb <= qc[ga] + qc[gb]) {
             total += ca + cb - qc[ga] - qc[gb];
             qc[ga] = ca;
@@ -1072,6 +1086,8 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
                 move_cnt(sb, pos[b], +1);
             }
         } else {
+            flip[a] = fa0;
+            flip[b] = fb0;
             std::swap(pos[a], pos[b]);
             std::swap(flip[a], flip[b]);
         }
