@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--buckets", type=int, default=8, help="config 5: launches per rank per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-paper-engine", action="store_true")
+    ap.add_argument("--no-lga", action="store_true", help="skip the full LGA docking-job measurement")
     return ap.parse_args()
 
 
@@ -640,6 +641,25 @@ def main():
         finally:
             ctx1.close()
 
+    # ---- NEXT-3: the whole Lamarckian GA docking job on this workload (Alg 1) with the
+    # paper's budgets (2.5e6 evaluations / 27 000 generations per run) -- the end-to-end
+    # number the paper quotes as us per evaluation (A100, real ligand: context only) ----
+    lga = None
+    if rank == 0 and not args.no_lga and not args.engine.startswith("paper"):
+        g_lga = start.clone()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        out = ctx.lga(lid, g_lga, n_runs, engine=args.engine, pop_size=w.pop, max_evals=2_500_000, max_gens=27000,
+                      ls_iters=w.iters, seed=1)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b)
+        ev = int(out["n_evals"].sum().item())
+        lga = {"runs": n_runs, "pop": w.pop, "budget": "2.5e6 evaluations or 27 000 generations per run (P:L57)",
+               "evaluations": ev, "generations_max": int(out["n_gens"].max().item()), "seconds": ms / 1e3,
+               "evals_per_s": ev / (ms / 1e3), "us_per_eval": ms * 1e3 / ev,
+               "best_energy_median": float(out["run_best"][:, 0].median().item())}
+
     # ---- paper-style block-per-pose engines, same workload (the self-built speedup denominator) ----
     paper = None
     if rank == 0 and not args.no_paper_engine and not args.engine.startswith("paper"):
@@ -697,6 +717,7 @@ def main():
                     "d2h_bytes_per_step": int((h_bestE.numel() + h_run.numel()) * 4)},
             "clocks": ck, "gpu_launches": 2 * args.steps,
             "config1_score_call": call1,
+            "lga": lga,
             "paper_baseline_engine": paper,
         }
         print(json.dumps(line), flush=True)

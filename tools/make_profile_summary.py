@@ -63,7 +63,8 @@ def main():
             for name, metric in (("issue_active_pct", "smsp__issue_active.avg.pct_of_peak_sustained_active"),
                                  ("l1tex_throughput_pct", "l1tex__throughput.avg.pct_of_peak_sustained_active"),
                                  ("warp_instructions", "smsp__inst_executed.sum"),
-                                 ("shared_wavefronts", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum")):
+                                 ("shared_wavefronts", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"),
+                                 ("tensor_pipe_pct", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active")):
                 if metric in s:
                     js["ls_kernel"][key][name] = float(s[metric][0])
         except (KeyError, ValueError):
