@@ -14,10 +14,12 @@ HEADERS = ["ad_internal.h", "ad_kernels.cuh"]
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17", "-ftz=true",
-    # no multiply-add contraction in ptxas: every FMA is explicit in the PTX (NVVM's),
-    # so both register-budget variants of a kernel round identically and results do
-    # not depend on which one a launch picks (+0.6 % instructions)
-    "-Xptxas", "--fmad=false",
+    # no multiply-add contraction, neither in NVVM (-fmad=false) nor in ptxas: every FMA
+    # is an explicit fmaf / fma / fma.f32x2 of the source, so every kernel variant
+    # (register budget, cherry-only twin, A14-instrumented) rounds identically and
+    # results do not depend on which one a launch picks.  (ptxas fuses a packed
+    # mul.f32x2 -> add/sub.f32x2 pair into FFMA2 even then: the packed code has none.)
+    "-fmad=false", "-Xptxas", "--fmad=false",
     "-Xcompiler", "-fPIC", "-shared",
 ]
 

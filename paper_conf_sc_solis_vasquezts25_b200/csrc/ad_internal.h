@@ -162,7 +162,9 @@ __host__ __device__ inline WarpScratch warp_scratch_layout(int32_t n_atoms, int3
     s.trig64 = o; o += 16 * n_tors;
     s.tw = o;    o += 32 * (6 + n_tors);  // per-gene gradient vectors (U, W) + rows
     s.genes = o; o += 4 * kMaxGenes;
-    o += 16 * 32;  // right after the genes: per-lane ADADELTA state (float4: E[g^2], E[dx^2], best, best E)
+    // right after the genes, narrow ligands (6 + T <= 32, one gene per lane): the per-lane
+    // ADADELTA state between updates (float4: E[g^2], E[dx^2], best gene, best E)
+    if (6 + n_tors <= 32) o += 16 * 32;
     s.part = o;  o += 16 * 32 * n_chunks;
     // the SIMT engine needs neither W nor D: its prefix sums overwrite the X and
     // slot-0 gradient rows the scan has just consumed (ad_kernels.cuh, a4-a5), so

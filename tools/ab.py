@@ -17,6 +17,7 @@ sys.path.insert(0, %r)
 from paper_conf_sc_solis_vasquezts25_b200 import ad, synth
 cfg, eng, w = int(sys.argv[1]), sys.argv[2], int(sys.argv[3])
 wl = synth.make_config(cfg)
+if os.environ.get("AB_ITERS"): wl.iters = int(os.environ["AB_ITERS"])  # shorter trajectories (A/B of code, not of trajectory luck)
 ctx = ad.Context(0); ctx.upload_grid(wl.grid); lid = ctx.upload_ligand(wl.ligands[0], wl.ff)
 start = torch.from_numpy(wl.genes).cuda(); g = start.clone()
 flush = torch.empty(64 * 1024 * 1024, device='cuda')
