@@ -63,7 +63,8 @@ struct LigSlot {
     int32_t block_scratch = 0;   // per block (baseline)
     int32_t n_atoms = 0, n_tors = 0;
     bool pkg = false;            // pre-decoded global-memory schedule (wide 128-register kernels)
-    bool smem_cherry = false;    // shared-memory cherries without PK_PRED: the cherry-only kernels (CH) run it
+    bool smem_cherry = false;    // shared-memory cherries without PK_PRED: the cherry-only kernels (CH = 1) run it
+    bool gm_cherry = false;      // global-memory cherries: the CH = 2 kernels run it
     float ff[FF_N] = {};         // LigHeader::ff (kernel parameters of every launch)
     bool live = false;
 };
@@ -1898,6 +1899,7 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
     s.n_tors = T;
     s.pkg = (W.h.off_pkg != 0 && 6 + T > 32) || (W.h.pk_flags & PK_GMEM);  // runs on the 128-register kernels
     s.smem_cherry = W.h.intra_mode == INTRA_SCATTER && W.h.off_pk != 0 && !(W.h.pk_flags & (PK_GMEM | PK_PRED));
+    s.gm_cherry = W.h.intra_mode == INTRA_SCATTER && W.h.off_pk != 0 && (W.h.pk_flags & PK_GMEM);
     memcpy(s.ff, H.ff, sizeof(s.ff));
     CUDA_TRY(cudaMalloc(&s.d_blob, W.buf.size()));
     CUDA_TRY(cudaMemcpy(s.d_blob, W.buf.data(), W.buf.size(), cudaMemcpyHostToDevice));
@@ -1964,14 +1966,16 @@ namespace {
 typedef void (*WarpKernelFn)(const KParams);
 struct WarpKernel {
     WarpKernelFn lo, hi;  // register budgets AD_WARP_MAXNREG / AD_WARP_MAXNREG_HI
-    WarpKernelFn lo_ch = nullptr, hi_ch = nullptr;  // cherry-only twins (CH; nullptr: none)
+    WarpKernelFn lo_ch = nullptr, hi_ch = nullptr;  // shared-memory-cherry-only twins (CH = 1; nullptr: none)
+    WarpKernelFn hi_gm = nullptr;                   // global-memory-cherry-only twin (CH = 2, 128 registers)
 };
 
 template <int E, bool GR, bool LS, bool W>
 WarpKernel wk() {
     return WarpKernel{k_warp_engine<E, GR, LS, AD_WARP_MAXNREG, W>, k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W>,
-                      k_warp_engine<E, GR, LS, AD_WARP_MAXNREG, W, false, true>,
-                      k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W, false, true>};
+                      k_warp_engine<E, GR, LS, AD_WARP_MAXNREG, W, false, 1>,
+                      k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W, false, 1>,
+                      k_warp_engine<E, GR, LS, AD_WARP_MAXNREG_HI, W, false, 2>};
 }
 
 // A14 instrumented LS kernels (ad_ls_params.phase_cycles): SIMT and TC engines
@@ -1979,8 +1983,9 @@ template <int E, bool W>
 WarpKernel wk_instr() {
     return WarpKernel{k_warp_engine<E, true, true, AD_WARP_MAXNREG, W, true>,
                       k_warp_engine<E, true, true, AD_WARP_MAXNREG_HI, W, true>,
-                      k_warp_engine<E, true, true, AD_WARP_MAXNREG, W, true, true>,
-                      k_warp_engine<E, true, true, AD_WARP_MAXNREG_HI, W, true, true>};
+                      k_warp_engine<E, true, true, AD_WARP_MAXNREG, W, true, 1>,
+                      k_warp_engine<E, true, true, AD_WARP_MAXNREG_HI, W, true, 1>,
+                      k_warp_engine<E, true, true, AD_WARP_MAXNREG_HI, W, true, 2>};
 }
 WarpKernel pick_instr_kernel(int engine, bool wide) {
     if (engine == AD_ENGINE_TC) return wide ? wk_instr<1, true>() : wk_instr<1, false>();
@@ -2069,12 +2074,15 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
     // ligands with global-memory schedules (pre-decoded places of wide ligands, streamed
     // cherry records) run the 128-register kernels, which alone carry those loops
     // (config 3: 121.0 ms vs 130.6 ms on the 80-register kernels' record-decoding loop)
-    bool pkg = L.pkg, ch = L.smem_cherry;
-    if (p.pose_ligand) for_each_launch_ligand(ctx, [&](const LigSlot& o) { pkg |= o.pkg; ch &= o.smem_cherry; });
+    bool pkg = L.pkg, ch = L.smem_cherry, gmc = L.gm_cherry;
+    if (p.pose_ligand)
+        for_each_launch_ligand(ctx, [&](const LigSlot& o) { pkg |= o.pkg; ch &= o.smem_cherry; gmc &= o.gm_cherry; });
     static const bool ch_on = !getenv("AD_NO_CH");  // A/B knob: generic kernels only
     if (ch && ch_on && kern.lo_ch) {  // every ligand of the launch runs shared-memory cherries: the cherry-only twins
         kern.lo = kern.lo_ch;
         kern.hi = kern.hi_ch;
+    } else if (gmc && ch_on && kern.hi_gm) {  // ... global-memory cherries (128-register kernels only)
+        kern.hi = kern.hi_gm;
     }
     // the decision depends on nothing else: cached (a config-1 score call is ~9 us of
     // kernel; the 64-candidate search must not add to it on every call)
