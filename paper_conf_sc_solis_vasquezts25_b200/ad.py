@@ -251,6 +251,17 @@ def ad_last_launch(ctx):
     return out
 
 
+def pair_loop_kind(ctx, lig) -> int:
+    """Inspection hook (not part of include/ad.h): 1 shared-memory cherries, 2 global-
+    memory cherries, 0 other pair loops (which kernel twins a launch of it can use)."""
+    try:
+        f = lib().adx_pair_loop
+    except AttributeError:
+        return 0
+    f.argtypes, f.restype = [C.c_void_p, C.c_int32], C.c_int32
+    return int(f(ctx, lig))
+
+
 # ---------------------------------------------------------------- convenience
 class Context:
     """One device context: grids + ligands uploaded once, many score / LS calls."""

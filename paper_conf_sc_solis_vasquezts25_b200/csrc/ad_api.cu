@@ -2522,6 +2522,15 @@ int32_t adx_debug_cherries(int32_t n_atoms, int32_t n_pairs, const int32_t* pair
     return AD_OK;
 }
 
+// Host-only inspection hook (not in include/ad.h): the pair loop a ligand runs --
+// 1 shared-memory cherries (the CH = 1 kernels), 2 global-memory cherries (CH = 2),
+// 0 any other (generic kernels), -1 bad id.  Launch buckets of one kind run the twins.
+int32_t adx_pair_loop(ad_context* ctx, int32_t lig) {
+    if (!ctx || lig < 0 || lig >= (int)ctx->ligs.size() || !ctx->ligs[lig].live) return -1;
+    const LigSlot& L = ctx->ligs[lig];
+    return L.smem_cherry ? 1 : L.gm_cherry ? 2 : 0;
+}
+
 // Host-only inspection hook (not in include/ad.h): register budget of the last
 // warp-engine launch (AD_WARP_MAXNREG or AD_WARP_MAXNREG_HI).
 int32_t adx_last_maxreg(ad_context* ctx) { return ctx ? ctx->last_maxreg : 0; }

@@ -72,17 +72,19 @@ def generate(spec, ks, processes=0):
     return dict(zip(ks, out))
 
 
-def make_buckets(mine, ligands, n_buckets):
-    """Split this rank's units into launch buckets: ordered by (wide ligand, pair
-    count) so a bucket never mixes >32-gene ligands with narrow ones (the wide
-    kernel variant would then run for all) and its footprint bound stays tight;
+def make_buckets(mine, ligands, n_buckets, kind=None):
+    """Split this rank's units into launch buckets: grouped by (wide ligand, pair-loop
+    kind) -- a bucket never mixes >32-gene ligands with narrow ones (the wide kernel
+    variant would then run for all) nor pair-loop kinds (a launch runs the specialised
+    kernel twins only when all its ligands share the kind; kind: ligand -> ad
+    .pair_loop_kind) -- ordered by pair count so the footprint bound stays tight, and
     cut at equal unit counts."""
-    order = sorted(mine, key=lambda kr: (6 + ligands[kr[0]].n_tors > 32, ligands[kr[0]].n_pairs, kr))
+    kind = kind or {}
+    key = lambda k: (6 + ligands[k].n_tors > 32, kind.get(k, 0))  # noqa: E731
+    order = sorted(mine, key=lambda kr: (key(kr[0]), ligands[kr[0]].n_pairs, kr))
     out = []
-    for wide in (False, True):
-        part = [u for u in order if (6 + ligands[u[0]].n_tors > 32) == wide]
-        if not part:
-            continue
+    for grp in sorted({key(k) for k, _ in mine}):
+        part = [u for u in order if key(u[0]) == grp]
         nb = max(1, round(n_buckets * len(part) / len(order)))
         out += [[part[i] for i in b] for b in np.array_split(np.arange(len(part)), min(nb, len(part))) if len(b)]
     return out
@@ -119,7 +121,8 @@ class Screen:
         t2 = time.perf_counter()
         dev = torch.device("cuda", torch.cuda.current_device())
         self.buckets = []
-        for us in make_buckets(mine, ligands, n_buckets):
+        kind = {k: ad.pair_loop_kind(ctx.h, self.lig_id[k]) for k in need}
+        for us in make_buckets(mine, ligands, n_buckets, kind):
             genes = np.concatenate([made[k][1][r * pop:(r + 1) * pop] for k, r in us])
             pl = np.repeat(np.array([self.lig_id[k] for k, _ in us], np.int32), pop)
             self.buckets.append({

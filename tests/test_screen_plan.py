@@ -59,6 +59,19 @@ def test_buckets_split_wide_and_narrow():
         assert max(ligs[k].n_pairs for k, _ in a) <= min(ligs[k].n_pairs for k, _ in c)
 
 
+def test_buckets_never_mix_pair_loop_kinds():
+    """Launches run the specialised kernel twins only when every ligand shares the pair
+    loop (ad.pair_loop_kind), so buckets are kind-pure; every unit lands once."""
+    spec = synth.ScreenSpec(n_ligands=48, runs=2, pop=4)
+    ligs = {k: spec.ligand(k) for k in range(48)}
+    mine = [(k, r) for k in range(48) for r in range(2)]
+    kind = {k: (1 if ligs[k].n_pairs < 500 else 2) if k % 7 else 0 for k in ligs}
+    buckets = screen.make_buckets(mine, ligs, 6, kind)
+    assert sorted(u for b in buckets for u in b) == sorted(mine)
+    for b in buckets:
+        assert len({kind[k] for k, _ in b}) == 1 and len({6 + ligs[k].n_tors > 32 for k, _ in b}) == 1
+
+
 def test_list_spec_slices_start_genes():
     spec = synth.ScreenSpec(n_ligands=3, runs=2, pop=4)
     ligs = [spec.ligand(k) for k in range(3)]
