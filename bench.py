@@ -356,7 +356,7 @@ def run_screen_bench(args):
     import torch
     import torch.distributed as dist
 
-    from paper_conf_sc_solis_vasquezts25_b200 import ad, report, screen, synth
+    from paper_conf_sc_solis_vasquezts25_b200 import ad, dist as addist, report, screen, synth
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -364,7 +364,7 @@ def run_screen_bench(args):
     local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        addist.init_process_group("nccl", torch.device("cuda", local))
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     cores = len(os.sched_getaffinity(0))
@@ -509,7 +509,7 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        addist.init_process_group("nccl", torch.device("cuda", local))
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
 

@@ -8,6 +8,7 @@ time first) on a cost model of one run's ADADELTA work.
 from __future__ import annotations
 
 import heapq
+import os
 
 
 def unit_cost(n_atoms: int, n_tors: int, n_pairs: int, pop: int, iters: int) -> float:
@@ -44,3 +45,18 @@ def gather_records(records, group=None):
     out = torch.empty((ws * src.shape[0],) + tuple(src.shape[1:]), dtype=src.dtype, device=src.device)
     dist.all_gather_into_tensor(out, src, group=group)
     return out.to(records.device)
+
+
+def init_process_group(backend: str, device=None):
+    """torch.distributed.init_process_group from the launcher's environment (RANK,
+    WORLD_SIZE, MASTER_ADDR/PORT) with a bounded collective timeout: a rank that dies
+    or hangs turns the one gather into an error after AD_DIST_TIMEOUT_S seconds
+    (default 600) instead of a silent hang (SURVEY §5 failure detection)."""
+    import datetime
+
+    import torch.distributed as dist
+    timeout = datetime.timedelta(seconds=float(os.environ.get("AD_DIST_TIMEOUT_S", "600")))
+    kw = {"timeout": timeout}
+    if device is not None and backend == "nccl":
+        kw["device_id"] = device
+    dist.init_process_group(backend, **kw)

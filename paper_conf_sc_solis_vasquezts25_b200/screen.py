@@ -12,6 +12,8 @@ energy, genes (stride)].
 """
 from __future__ import annotations
 
+import os
+
 import numpy as np
 
 from . import dist as addist
@@ -150,21 +152,38 @@ class Screen:
             b["host"] = b["start"].cpu().pin_memory()
         return sum(b["host"].numel() * 4 for b in self.buckets)
 
-    def step(self, n_evals=None, gather=True, from_host=False):
+    def step(self, n_evals=None, gather=True, from_host=False, ckpt_dir=None, rank=0):
         """Restore the start genotypes (device copy, or from the pinned host copies
         with from_host), run every bucket's LS launch, write the unit records; then
         (world > 1) gather them.  Enqueued on the current stream; returns the
-        (gathered) record tensor."""
+        (gathered) record tensor.
+
+        ckpt_dir (screen resilience): every finished bucket's records are
+        written to ckpt_dir/rank<rank>_bucket<i>.npy (synchronously, atomic rename), and
+        a bucket whose file exists is not launched again but read back -- a screen
+        restarted after a crash or preemption resumes at its first unfinished bucket."""
+        import torch
         ad = self.ad
         row = 0
-        for b in self.buckets:
+        for i, b in enumerate(self.buckets):
+            n = len(b["units"])
+            path = os.path.join(ckpt_dir, f"rank{rank}_bucket{i}.npy") if ckpt_dir else None
+            if path and os.path.exists(path):
+                saved = torch.from_numpy(np.load(path)).to(self.rec.device)
+                if tuple(saved.shape) == (n, self.rec.shape[1]) and torch.equal(saved[:, :2], b["ids"]):
+                    self.rec[row:row + n] = saved
+                    row += n
+                    continue
             b["genes"].copy_(b["host"] if from_host else b["start"], non_blocking=True)
             ad.ad_set_launch_ligands(self.ctx.h, b["lig_ids"])
             ad.ad_local_search(self.ctx.h, b["bound"], b["pl"], b["genes"], b["bE"], b["rb"], n_evals,
                                max_iters=self.iters, pop_per_run=self.pop, engine=ad.ENGINES[self.engine])
-            n = len(b["units"])
             self.rec[row:row + n, :2] = b["ids"]
             self.rec[row:row + n, 2:] = b["rb"]
+            if path:
+                os.makedirs(ckpt_dir, exist_ok=True)
+                np.save(path + ".tmp.npy", self.rec[row:row + n].cpu().numpy())  # (synchronises the stream)
+                os.replace(path + ".tmp.npy", path)
             row += n
         ad.ad_set_launch_ligands(self.ctx.h, None)
         return addist.gather_records(self.rec) if gather else self.rec
@@ -176,15 +195,16 @@ class Screen:
 
 
 def run_screen(ctx, grid, ff, ligands, start_genes, runs, pop, iters, rank=0, world=1, engine="simt",
-               n_buckets=4, stream_sync=True):
+               n_buckets=4, stream_sync=True, ckpt_dir=None):
     """One screen: start_genes [n_ligands * runs * pop, stride] host array
     (ligand-major, run, pop).  Returns (records [world * n_rec, 3 + stride] torch
-    tensor on the rank's device, units list)."""
+    tensor on the rank's device, units list).  ckpt_dir: per-bucket result files,
+    resume (Screen.step)."""
     import torch
     s = Screen(ctx, ListSpec(grid, ligands, start_genes, runs, pop, iters), ff, rank=rank, world=world,
                engine=engine, n_buckets=n_buckets)
     try:
-        rec = s.step()
+        rec = s.step(ckpt_dir=ckpt_dir, rank=rank)
         if stream_sync:
             ctx.sync()  # device-side argument errors (pose_ligand, footprint, stride) raise here
         return rec, s.units

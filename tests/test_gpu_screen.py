@@ -45,3 +45,38 @@ def test_screen_matches_single_ligand_runs():
                 assert bad.size == 0, (k, r, L.n_tors, bad, got[(k, r)][bad], rb[r][bad])
     finally:
         ctx.close()
+
+
+def test_screen_checkpoint_resume(tmp_path):
+    """Screen resilience: with ckpt_dir every finished bucket's records are
+    saved; a resumed screen launches only the buckets without a file (counted by the
+    evaluation counter) and returns the same records bit for bit."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import os
+
+    from paper_conf_sc_solis_vasquezts25_b200 import ad, screen
+    grid = synth.make_grid(5200, 40, synth.TYPESETS[8], 800)
+    ff = synth.FFParams()
+    ligs = [synth.make_ligand(900 + k, 24 + 3 * k, k % 5, 8) for k in range(6)]
+    runs, pop, iters, stride = 2, 8, 10, 16
+    genes = np.concatenate([synth.make_genotypes(k, runs * pop, L.n_tors, grid, stride=stride, frac=0.3)
+                            for k, L in enumerate(ligs)])
+    ctx = ad.Context(0)
+    try:
+        spec = screen.ListSpec(grid, ligs, genes, runs, pop, iters)
+        s = screen.Screen(ctx, spec, ff, n_buckets=3)
+        ev = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ck = str(tmp_path / "ckpt")
+        rec0 = s.step(n_evals=ev, gather=False, ckpt_dir=ck).cpu().numpy().copy()
+        full = int(ev.item())
+        files = sorted(os.listdir(ck))
+        assert len(files) == len(s.buckets) and full == len(s.units) * pop * iters
+        os.remove(os.path.join(ck, files[0]))          # bucket 0 "lost"
+        ev.zero_()
+        rec1 = s.step(n_evals=ev, gather=False, ckpt_dir=ck).cpu().numpy()
+        assert 0 < int(ev.item()) < full                # only bucket 0 ran again
+        assert np.array_equal(rec0, rec1)
+        s.close()
+    finally:
+        ctx.close()
