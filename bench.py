@@ -548,15 +548,17 @@ def main():
         if world > 1:
             addist.gather_records(run_best)
 
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
+    nvtx = torch.cuda.nvtx  # ranges on the Nsight timeline; libad adds one per ABI call
+    with nvtx.range("bench.warmup"):
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     ev_step = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     ev_kern = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     n_evals.zero_()
-    with ClockSampler(local) as clocks:
+    with ClockSampler(local) as clocks, nvtx.range("bench.timed"):
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
@@ -584,6 +586,7 @@ def main():
     h_bestE = torch.empty(n).pin_memory()
     h_run = torch.empty(n_runs, 1 + stride).pin_memory()
     e2e_ev = []
+    nvtx.range_push("bench.e2e")
     for k in range(max(2, args.steps)):
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         flush.fill_(float(k))
@@ -596,6 +599,7 @@ def main():
         b.record(stream)
         e2e_ev.append((a, b))
     torch.cuda.synchronize()
+    nvtx.range_pop()
     e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_ev) / len(e2e_ev)
     e2e_t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
     if world > 1:

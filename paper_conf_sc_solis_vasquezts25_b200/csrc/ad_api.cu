@@ -10,6 +10,7 @@
 //               per-pair desolvation prefactors, (cA, cB, r0, n) table.
 // Launches pick warps-per-CTA from the occupancy calculator.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges cost a pointer check unless a tool is attached
 
 #include <algorithm>
 #include <array>
@@ -27,6 +28,16 @@
 #include "ad.h"
 #include "ad_internal.h"
 #include "ad_kernels.cuh"
+
+namespace {
+// NVTX range over one ABI call (Nsight Systems / Compute timelines; SURVEY §5 tracing)
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+}  // namespace
 
 using namespace adk;
 
@@ -1452,6 +1463,7 @@ int32_t ad_context_destroy(ad_context* ctx) {
 
 int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* d, const float* maps, int32_t maps_on_device,
                         void* stream) {
+    NvtxRange nvtx_range("ad_upload_grids");
     if (!ctx || !d || !maps) return fail(AD_ERR_INVALID_ARG, "null argument");
     if (d->nx < 2 || d->ny < 2 || d->nz < 2) return fail(AD_ERR_INVALID_ARG, "grid needs >= 2 points per axis");
     if (d->n_maps < 3 || d->n_maps > AD_MAX_MAPS) return fail(AD_ERR_LIMIT, "n_maps %d not in [3,%d]", d->n_maps, AD_MAX_MAPS);
@@ -1536,6 +1548,7 @@ int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* d, const float* map
 }
 
 int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id* out) {
+    NvtxRange nvtx_range("ad_upload_ligand");
     if (!ctx || !d || !out) return fail(AD_ERR_INVALID_ARG, "null argument");
     *out = -1;
     if (!ctx->has_grid) return fail(AD_ERR_STATE, "upload grids before ligands");
@@ -2183,6 +2196,7 @@ extern "C" {
 int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses,
                        const float* genes, int32_t geno_stride, float* energy, float* grad, float* aux,
                        void* stream) {
+    NvtxRange nvtx_range("ad_score_poses");
     if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
     if (n_poses > 0 && !energy) return fail(AD_ERR_INVALID_ARG, "energy is NULL");
     if (pose_ligand) {
@@ -2208,6 +2222,7 @@ int32_t ad_score_poses(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_li
 int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_ligand, int32_t n_poses, float* genes,
                         int32_t geno_stride, float* best_energy, float* run_best, int64_t* n_evals,
                         const ad_ls_params* prm, void* stream) {
+    NvtxRange nvtx_range("ad_local_search");
     if (int32_t rc = common_checks(ctx, lig, n_poses, genes, geno_stride)) return rc;
     if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
     if (prm->max_iters < 1) return fail(AD_ERR_INVALID_ARG, "max_iters must be >= 1");
@@ -2292,6 +2307,7 @@ int32_t ad_local_search(ad_context* ctx, ad_ligand_id lig, const int32_t* pose_l
 int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* genes, int32_t geno_stride,
                    float* energies, float* run_best, int64_t* n_evals, int32_t* n_gens, const ad_lga_params* prm,
                    void* stream) {
+    NvtxRange nvtx_range("ad_lga_run");
     if (!prm) return fail(AD_ERR_INVALID_ARG, "params is NULL");
     const int pop = prm->pop_size;
     if (n_runs < 0 || pop < 2 || pop > 4096) return fail(AD_ERR_INVALID_ARG, "need n_runs >= 0, 2 <= pop_size <= 4096");
@@ -2420,6 +2436,7 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
 
 int32_t ad_reduce_blocks(ad_context* ctx, int32_t engine, int32_t n_blocks, int32_t n_partials, int32_t n_comp,
                          const float* partials, float* out, void* stream) {
+    NvtxRange nvtx_range("ad_reduce_blocks");
     if (!ctx || !partials || !out) return fail(AD_ERR_INVALID_ARG, "null argument");
     if (n_blocks < 0) return fail(AD_ERR_INVALID_ARG, "n_blocks < 0");
     if (n_partials < 32 || n_partials > 1024 || n_partials % 32) return fail(AD_ERR_INVALID_ARG, "n_partials %d", n_partials);
