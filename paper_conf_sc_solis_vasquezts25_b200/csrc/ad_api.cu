@@ -2407,10 +2407,19 @@ int32_t ad_lga_run(ad_context* ctx, ad_ligand_id lig, int32_t n_runs, float* gen
         // LS(population): compacted list, gather, ADADELTA, scatter back (Lamarckian)
         k_ga_ls_select<<<n_runs, 128, 0, st>>>(G, d_done, (uint32_t)gen, d_list, d_cnt, d_per);
         LGA_TRY(cudaGetLastError());
+        // the LS launch is shaped for the individuals actually selected (ls_rate of the
+        // population): read back the count first, so the CTAs spread over every SM instead
+        // of a grid sized for the whole population whose tail CTAs exit at once (config 2,
+        // ls_rate 0.8: ~2400 of 3000 poses on ~113 of 148 SMs)
+        int32_t h_cnt = 0;
+        LGA_TRY(cudaMemcpyAsync(&h_cnt, d_cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
         const int rb = std::min(65535, (n_ind * S + 255) / 256);
         k_ga_rows<<<rb, 256, 0, st>>>(d_list, d_cnt, S, cur, d_lsg, false, nullptr, nullptr);
         LGA_TRY(cudaGetLastError());
-        if (int32_t rc = launch_warp(ctx, L, ls_kern, lp, ls.warps_per_cta, st, tc)) { cleanup(); return rc; }
+        LGA_TRY(cudaStreamSynchronize(st));
+        lp.n_poses = std::min(std::max(h_cnt, 0), n_ind);
+        if (lp.n_poses > 0)
+            if (int32_t rc = launch_warp(ctx, L, ls_kern, lp, ls.warps_per_cta, st, tc)) { cleanup(); return rc; }
         k_ga_rows<<<rb, 256, 0, st>>>(d_list, d_cnt, S, d_lsg, cur, true, d_lse, energies);
         LGA_TRY(cudaGetLastError());
         k_ga_update<<<(n_runs + 127) / 128, 128, 0, st>>>(n_runs, pop, ls.max_iters, prm->max_evals, prm->max_gens,
