@@ -1136,19 +1136,26 @@ CherrySchedule schedule_cherries(int n_idx, const std::vector<int>& pi, const st
 // (cherry_rows_fit).
 struct CherryRecords {
     std::vector<uint4> a;
-    std::vector<float4> b, c;
+    std::vector<float4> b;
+    std::vector<float4> c;   // 48-B records (shared-memory cherries): (r0, r0', -cC, -cC')
+    std::vector<float2> c2;  // 40-B records (global-memory cherries): (r0, r0')
     int n_spare = 8;
 };
 bool cherry_rows_fit(int npad, int K) { return npad + 8 <= 256 && K * npad + 8 <= 256; }
 int cherry_max_slots(int npad) { return npad + 8 <= 256 ? std::min(8, (256 - 8) / npad) : 0; }
 
+// compact: the 40-B record of the global-memory cherry loop (intra_cherry_gm): each pair's one
+// nonzero dispersion coefficient in b, its 12-10 flag in a.x bits 24-25 (config 3: 108.2 ->
+// 104.7 ms per LS launch, the loop being L1-bound; bit-identical).  The shared-memory loop keeps
+// the 48-B record: its 80-register kernel pays more for the selects than it saves (2.99 -> 3.02 ms).
 CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector<int>& ptp,
-                            const std::vector<float4>& tp, const std::vector<float>& pdsv, bool distinct) {
+                            const std::vector<float4>& tp, const std::vector<float>& pdsv, bool distinct,
+                            bool compact) {
     CherryRecords R;
     const size_t n = (size_t)S.steps * 32;
     R.a.resize(n);
     R.b.resize(n);
-    R.c.resize(n);
+    if (compact) R.c2.resize(n); else R.c.resize(n);
     const int K = S.slots;
     uint64_t step_used[4] = {0, 0, 0, 0};  // dummy rows (0..255) taken in the current step
     for (size_t q0 = 0; q0 < n; q0 += 8) {  // one quarter-warp
@@ -1187,6 +1194,7 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector
                 dummy(0);
             }
             float cA[2], cB[2], cC[2], r0[2], dsv[2];
+            bool hbk[2] = {false, false};
             for (int k = 0; k < 2; ++k) {
                 if (L.c >= 0 && L.e[k] >= 0) {
                     xr[1 + k] = (uint32_t)L.e[k];
@@ -1196,6 +1204,7 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector
                     cA[k] = t.x;
                     cB[k] = hb ? 0.f : -t.y;  // negated: pair_term2 takes -cB, -cC (no negations in the loop)
                     cC[k] = hb ? -t.y : 0.f;
+                    hbk[k] = hb;
                     r0[k] = t.z;
                     dsv[k] = pdsv[L.p[k]];
                 } else {
@@ -1210,10 +1219,21 @@ CherryRecords pack_cherries(const CherrySchedule& S, int npad, const std::vector
             memcpy(&d1, &dsv[1], 4);
             // a.y bits 24-26: the centre / end 0 / end 1 is empty (PK_PRED: the kernel skips its store)
             const uint32_t fl = (L.c < 0 ? 1u : 0u) | (L.c < 0 || L.e[0] < 0 ? 2u : 0u) | (L.c < 0 || L.e[1] < 0 ? 4u : 0u);
-            R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16),
-                                gr[0] | (gr[1] << 8) | (gr[2] << 16) | (fl << 24), d0, d1);
-            R.b[q] = make_float4(cA[0], cA[1], cB[0], cB[1]);
-            R.c[q] = make_float4(r0[0], r0[1], cC[0], cC[1]);
+            if (compact) {
+                // a.x bits 24-25: pair k is a 12-10 (H-bond) pair, whose one nonzero dispersion
+                // coefficient (-cC) then rides in b where a 12-6 pair's -cB goes (the kernel
+                // rebuilds the (-cB, -cC) operands with selects: the same values, 8 B less)
+                const uint32_t hbf = (hbk[0] ? 1u : 0u) | (hbk[1] ? 2u : 0u);
+                R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16) | (hbf << 24),
+                                    gr[0] | (gr[1] << 8) | (gr[2] << 16) | (fl << 24), d0, d1);
+                R.b[q] = make_float4(cA[0], cA[1], hbk[0] ? cC[0] : cB[0], hbk[1] ? cC[1] : cB[1]);
+                R.c2[q] = make_float2(r0[0], r0[1]);
+            } else {
+                R.a[q] = make_uint4(xr[0] | (xr[1] << 8) | (xr[2] << 16),
+                                    gr[0] | (gr[1] << 8) | (gr[2] << 16) | (fl << 24), d0, d1);
+                R.b[q] = make_float4(cA[0], cA[1], cB[0], cB[1]);
+                R.c[q] = make_float4(r0[0], r0[1], cC[0], cC[1]);
+            }
         }
     }
     return R;
@@ -1824,19 +1844,20 @@ int32_t ad_upload_ligand(ad_context* ctx, const ad_ligand_desc* d, ad_ligand_id*
             // cherry_gm, left in global memory).  Distinct dummy rows when they fit the
             // 8-bit row indices and at most 32 spare rows (512 B per warp), else shared
             // dummies with predicated stores (PK_PRED).
-            CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, true);
+            CherryRecords cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, true, cherry_gm);
             h.pk_flags = cherry_gm ? PK_GMEM : 0;
             // (global-memory cherries always take the predicated loop: measured faster than
             // distinct dummies on config 3, 114.1 vs 120.4 ms per LS launch)
             if (cherry_gm || cs.slots * h.n_pad + cr.n_spare > 256 || cr.n_spare > 32) {
-                cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, false);
+                cr = pack_cherries(cs, h.n_pad, ptp, tp, pd, false, cherry_gm);
                 h.pk_flags |= PK_PRED;
             }
             o.ws = warp_scratch_layout(N, T, h.n_slots, own.C, cr.n_spare);
             h.off_tp = h.off_prec = h.off_pdsv = h.off_pkg = 0;
             h.off_pk = B.put(cr.a.data(), sizeof(uint4) * cr.a.size());
             B.put(cr.b.data(), sizeof(float4) * cr.b.size());
-            B.put(cr.c.data(), sizeof(float4) * cr.c.size());
+            if (cherry_gm) B.put(cr.c2.data(), sizeof(float2) * cr.c2.size());
+            else B.put(cr.c.data(), sizeof(float4) * cr.c.size());
             h.pairs_gmem = cherry_gm ? 1 : 0;  // (cherry_gm: records after the staged prefix)
             h.blob_bytes = (int32_t)B.buf.size();
             h.stage_bytes = cherry_gm ? h.off_pk : h.blob_bytes;

@@ -27,7 +27,8 @@
 //                           lane l reads copy l%8 -> conflict-free 128-bit lookups
 //   pka     u32x4  [R*32]   (cherry schedule, off_pk != 0: INTRA_SCATTER with the schedule
 //   pkb     f32x4  [R*32]   in shared memory; R = n_rounds cherry steps of 32 lanes, each lane
-//   pkc     f32x4  [R*32]   two pairs sharing a centre atom) -- see intra_cherry in ad_kernels.cuh
+//   pkc     f32x4  [R*32]   two pairs sharing a centre atom) -- see intra_cherry in ad_kernels.cuh;
+//           global-memory cherries (PK_GMEM): pkc f32x2 [R*32] (40-B records, pack_cherries compact)
 //           The warp engine stages the whole blob; the paper-style baseline stages
 //           [0, off_pk) (prec / pdsv / tp), its footprint unchanged.
 //
