@@ -1502,10 +1502,14 @@ int32_t ad_upload_grids(ad_context* ctx, const ad_grid_desc* d, const float* map
     const int nt = d->n_maps - 2;
     const float* E = h.data() + (size_t)nt * vol;
     const float* D = h.data() + (size_t)(nt + 1) * vol;
-    // Cell records (3 x 256-bit loads per atom, 8x the map bytes) when they stay
-    // comfortably L2-resident, else x-pair records (8 loads per atom, 2x bytes).
+    // Cell records (3 x 256-bit loads per atom, 8x the map bytes) up to 1 GiB of records,
+    // else x-pair records (8 loads per atom, 2x bytes).  The poses of a search stay in the
+    // pocket, so the cells they touch are a small part of the grid and L2-resident even
+    // when the whole record set is not: config 3 (96^3, 8 type maps: 283 MB of cell
+    // records) runs 104.7 (x-pair) -> 98.6 ms per LS launch with cells (its LS kernel is
+    // L1-bound, and a cell gather is 3 wide loads instead of 8)
     const size_t cell_bytes = vol * ((size_t)nt * 32 + 64);
-    int layout = cell_bytes <= ((size_t)64 << 20) ? 1 : 0;
+    int layout = cell_bytes <= ((size_t)1 << 30) ? 1 : 0;
     if (const char* e = getenv("AD_GRID_LAYOUT")) layout = strcmp(e, "cell") == 0 ? 1 : strcmp(e, "xpair") == 0 ? 0 : layout;
     if (ctx->d_tmap) { cudaFree(ctx->d_tmap); ctx->d_tmap = nullptr; }
     if (ctx->d_ed) { cudaFree(ctx->d_ed); ctx->d_ed = nullptr; }
