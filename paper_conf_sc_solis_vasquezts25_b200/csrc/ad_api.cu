@@ -2166,10 +2166,15 @@ int32_t launch_warp(ad_context* ctx, LigSlot L, WarpKernel kern, KParams& p, int
             const double g1 = 1.0 - 0.48;
             double cost = (double)full * std::pow((double)active, g1) + (rem ? std::pow((double)(rem * w), g1) : 0.0);
             if (v) cost *= 0.85;
+            const size_t sm_smem = (size_t)std::min<long>(blocks, per_sm) * smem;  // in use on the busiest SM
+            // shared memory in use is L1 taken from the grid gathers, the streamed records
+            // and the spills: +10 % cost for a full SM (config 3, W = 2 / 4 / 8 / 16 -> 191 /
+            // 159 / 143 / 135 KB per SM: 98.6 / 97.2 / 96.4 / 102.3 ms per LS launch; the
+            // wave model alone picked W = 2)
+            cost *= 1.0 + 0.1 * (double)sm_smem / (double)std::max(ctx->max_smem_optin, 1);
             if (debug_launch)
                 fprintf(stderr, "[libad] regs=%d w=%d smem=%zu blocks/SM=%d active=%d ctas=%ld per_sm=%ld cost=%.3f\n",
                         v ? AD_WARP_MAXNREG_HI : AD_WARP_MAXNREG, w, smem, blocks, active, ctas, per_sm, cost);
-            const size_t sm_smem = (size_t)std::min<long>(blocks, per_sm) * smem;  // in use on the busiest SM
             const bool better = cost < pick.cost - 1e-9 ||
                                 (cost < pick.cost + 1e-9 && (sm_smem < pick.sm_smem || (sm_smem == pick.sm_smem && active > pick.active)));
             if (better) pick = Cand{w, active, cost, sm_smem, smem, k};
